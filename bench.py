@@ -1,0 +1,312 @@
+#!/usr/bin/env python
+"""bench.py — NW GCUPS + HBM roofline of the B200 wavefront (BASELINE.json metric).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C] [--tile B] [--impl ours|reference]
+
+One step = one pass of the whole hot path (one nw_fill / nw_fill_batch call = ONE kernel launch)
+over the config's synthetic input, resident in HBM.  Defaults: N=1 -> config 3 (n=32768, the
+headline, BASELINE.json configs[2]); N>1 (torchrun) -> config 4 (4096 independent n=2048 pairs
+split contiguously over the ranks, no collective on the data path).  Prints ONE JSON line on
+rank 0.  Inputs (8.6 GB at config 3) are far larger than the 126 MB L2, so no flush is needed.
+
+--impl reference times the CPU oracle (oracle/nw_ref.c, single-threaded) on a bounded sample of
+the same workload on the host cores (rank 0 only), as the driver's reference arm.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+CONFIGS = {
+    1: dict(workload="nw_n1024_p10_tile16", n=1024, batch=1, tile=16),
+    2: dict(workload="nw_n16384_p10", n=16384, batch=1, tile=64),
+    3: dict(workload="nw_n32768_p10", n=32768, batch=1, tile=0),
+    4: dict(workload="nw_batch4096_n2048_p10", n=2048, batch=4096, tile=0),
+}
+PENALTY = 10
+METRIC = "NW GCUPS (interior cell updates / s), bit-exact vs CPU oracle"
+
+
+def env_int(k, d):
+    try:
+        return int(os.environ.get(k, d))
+    except ValueError:
+        return d
+
+
+class Clocks:
+    """nvidia-smi sampler during the timed region (clocks + throttle reasons)."""
+
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index, self.rows, self._stop = index, [], threading.Event()
+        self._t = threading.Thread(target=self._run, daemon=True)
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                out = subprocess.run(["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
+                                      "--format=csv,noheader,nounits"], capture_output=True, text=True,
+                                     timeout=5).stdout.strip()
+                if out:
+                    self.rows.append([x.strip() for x in out.split(",")])
+            except Exception:
+                pass
+            self._stop.wait(0.2)
+
+    def __enter__(self):
+        self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        self._t.join(timeout=10)
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"], "samples": 0}
+        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in self.rows for i in range(4) if len(r) > 4 + i and r[4 + i] == "Active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.rows)}
+
+
+def measured_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            j = json.load(f)
+        return float(j["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, burst copy)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def ncu_traffic(workload, tile):
+    """DRAM bytes per launch of the dominant kernel from the committed ncu --set full summary."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
+            j = json.load(f)
+        return j.get(f"{workload}/tile{tile}")
+    except Exception:
+        return None
+
+
+def cpu_baseline(cfg, gpu_last_row=None):
+    """The oracle as it stands (single-threaded C) on a bounded sample of the workload."""
+    import numpy as np
+
+    import inputs
+    import oracle
+    n, p = cfg["n"], PENALTY
+    if cfg["batch"] == 1:
+        # whole matrix, streamed (O(n) memory): rows generated block by block from the same seed
+        a, b = inputs.gen_pair(n, inputs.SEED)
+        row0 = -np.arange(n + 1, dtype=np.int32) * p
+        st = oracle.NwRefStream(n, p, row0)
+        t_or = 0.0
+        rows_done = 0
+        budget = float(os.environ.get("NW_CPU_BASELINE_S", "25"))
+        last = None
+        for i0 in range(1, n + 1, 1024):
+            i1 = min(n + 1, i0 + 1024)
+            blk = inputs.build_ref_block(a, b, i0, i1)
+            col0 = (-np.arange(i0, i1, dtype=np.int64) * p).astype(np.int32)
+            t = time.perf_counter()
+            out = st.rows(blk, col0, want_out=(i1 == n + 1))
+            t_or += time.perf_counter() - t
+            rows_done = i1 - 1
+            if i1 == n + 1:
+                last = out[-1]
+            if t_or > budget:
+                break
+        st.close()
+        cells = rows_done * n
+        sample = f"rows 1..{rows_done} of the n={n} matrix (streaming oracle, {cells:.3e} cells)"
+        exact = None
+        if last is not None and gpu_last_row is not None:
+            exact = bool(np.array_equal(last, gpu_last_row))
+        return {"value": cells / t_or / 1e9, "unit": "GCUPS", "cores": 1, "kind": "oracle",
+                "sample": sample, "seconds": t_or, "last_row_bit_exact": exact}
+    # batch: the first pairs of the batch, one by one
+    t_or, cells, k = 0.0, 0, 0
+    budget = float(os.environ.get("NW_CPU_BASELINE_S", "15"))
+    while t_or < budget and k < cfg["batch"]:
+        s, r = inputs.make_problem(n, p, seed=inputs.pair_seed(k))
+        t = time.perf_counter()
+        oracle.nw_ref(s, r, p)
+        t_or += time.perf_counter() - t
+        cells += n * n
+        k += 1
+    return {"value": cells / t_or / 1e9, "unit": "GCUPS", "cores": 1, "kind": "oracle",
+            "sample": f"first {k} of {cfg['batch']} pairs (n={n})", "seconds": t_or}
+
+
+def run_reference(args, cfg, rank):
+    if rank != 0:
+        return
+    import oracle
+    oracle.build()
+    steps = []
+    # each step is a bounded sample so the whole --steps K --warmup W run stays within minutes
+    os.environ["NW_CPU_BASELINE_S"] = str(min(25.0, 150.0 / (args.warmup + args.steps)))
+    for _ in range(args.warmup + args.steps):
+        steps.append(cpu_baseline(dict(cfg), None))
+    timed = steps[args.warmup:]
+    v = statistics.mean(s["value"] for s in timed)
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "GCUPS", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "higher_is_better": True, "dtype": "int32",
+            "data": "synthetic", "config": {"workload": cfg["workload"], "n": cfg["n"], "batch": cfg["batch"],
+                                            "penalty": PENALTY},
+            "cpu_baseline": {"value": v, "unit": "GCUPS", "cores": 1, "kind": "oracle",
+                             "sample": timed[0]["sample"]},
+            "e2e": {"value": v, "unit": "GCUPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", type=int, default=0)
+    ap.add_argument("--tile", type=int, default=-1)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--no-cpu", action="store_true")
+    args = ap.parse_args()
+    world = env_int("WORLD_SIZE", 1)
+    rank = env_int("RANK", 0)
+    local_rank = env_int("LOCAL_RANK", 0)
+    cfg_id = args.config or (3 if world == 1 else 4)
+    cfg = dict(CONFIGS[cfg_id])
+    if args.tile >= 0:
+        cfg["tile"] = args.tile
+    args.warmup = max(args.warmup, 3)
+    if args.impl == "reference":
+        return run_reference(args, cfg, rank)
+
+    import numpy as np
+    import torch
+
+    import inputs
+    import paper_conf_sc_munksgaardhso22_b200 as nwb
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=dev)
+    n, p, tile = cfg["n"], PENALTY, cfg["tile"]
+    B = cfg["batch"]
+    if B > 1:
+        per = B // world
+        lo = rank * per
+        hi = B if rank == world - 1 else lo + per
+        nb = hi - lo
+        S = torch.empty((nb, n + 1, n + 1), dtype=torch.int32, device=dev)
+        R = torch.empty((nb, n + 1, n + 1), dtype=torch.int32, device=dev)
+        for k in range(nb):
+            inputs.device_problem(n, p, seed=inputs.pair_seed(lo + k), device=dev, score=S[k], ref=R[k])
+
+        def step():
+            nwb.nw_fill_batch(S, R, p, tile)
+        cells_local = nb * n * n
+    else:
+        S, R = inputs.device_problem(n, p, device=dev)
+
+        def step():
+            nwb.nw_fill(S, R, p, tile)
+        cells_local = n * n
+    torch.cuda.synchronize()
+    stream = torch.cuda.current_stream()
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    with Clocks(local_rank) as clk:
+        time.sleep(0.3)
+        torch.cuda.synchronize()
+        t0 = torch.cuda.Event(enable_timing=True)
+        t1 = torch.cuda.Event(enable_timing=True)
+        t0.record(stream)
+        for e0, e1 in ev:
+            e0.record(stream)
+            step()
+            e1.record(stream)
+        t1.record(stream)
+        torch.cuda.synchronize()
+    total_ms = t0.elapsed_time(t1)
+    per_launch = [e0.elapsed_time(e1) for e0, e1 in ev]
+    if world > 1:
+        tt = torch.tensor([total_ms], device=dev)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        total_ms = float(tt.item())
+    cells_total = cells_local if world == 1 else B * n * n
+    ms_per_step = total_ms / args.steps
+    value = cells_total / (ms_per_step * 1e-3) / 1e9
+    # roofline of the (only) kernel: 8 algorithmic bytes per interior cell (ref read + score write)
+    kern_ms = statistics.mean(per_launch)
+    achieved = 8.0 * cells_local / (kern_ms * 1e-3) / 1e9
+    peak, peak_src = measured_peaks()
+    roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+            "traffic": ncu_traffic(cfg["workload"], tile), "peak_source": peak_src,
+            "algorithmic_bytes_per_launch": 8 * cells_local,
+            "kernel": "nw_strip_kernel<%d>" % (4 if tile in (0, 128) else 2),
+            "kernel_ms_mean": kern_ms, "kernel_ms_median": statistics.median(per_launch)}
+    out = {"metric": METRIC, "value": value, "unit": "GCUPS", "n_gpus": world, "steps": args.steps,
+           "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+           "scaling": "strong" if world > 1 else "weak", "vs_baseline": None, "dtype": "int32",
+           "data": "synthetic (splitmix64 seq 7, BLOSUM62 ref, global-alignment borders)",
+           "config": {"workload": cfg["workload"], "n": n, "batch": B, "penalty": p, "tile": tile,
+                      "band_width": nwb.nw_band_width(tile), "pairs_per_rank": B // world if B > 1 else 1,
+                      "l2": "inputs %.1f GB >> 126 MB L2 (no flush needed)" % (8.0 * (n + 1) ** 2 * B / 1e9),
+                      "parallelism": f"dp{world}" if world > 1 else "single"},
+           "roofline": roof, "gpu_launches": args.steps * nwb.nw_launch_count(0, n, tile),
+           "clocks": clk.summary()}
+    # ---- e2e through the public C ABI with host buffers (H2D + kernel + D2H inside the timing)
+    if B == 1 and args.e2e_steps > 0:
+        hs = torch.empty((n + 1, n + 1), dtype=torch.int32, pin_memory=True)
+        hr = torch.empty((n + 1, n + 1), dtype=torch.int32, pin_memory=True)
+        hr.copy_(R.cpu())
+        hs[0].copy_(S[0].cpu())
+        hs[:, 0].copy_(S[:, 0].cpu())
+        hs_np, hr_np = hs.numpy(), hr.numpy()
+        nwb.nw_fill_host(hs_np, hr_np, p, tile, local_rank)       # warm-up (allocations)
+        t = time.perf_counter()
+        for _ in range(args.e2e_steps):
+            nwb.nw_fill_host(hs_np, hr_np, p, tile, local_rank)
+        e2e_s = (time.perf_counter() - t) / args.e2e_steps
+        out["e2e"] = {"value": cells_local / e2e_s / 1e9, "unit": "GCUPS",
+                      "h2d_bytes_per_step": 4 * (n + 1) ** 2 + 4 * (2 * n + 1),
+                      "d2h_bytes_per_step": 4 * (n + 1) ** 2, "ms_per_step": e2e_s * 1e3,
+                      "api": "nw_fill_host (pinned host buffers)"}
+        out["gpu_launches_e2e"] = args.e2e_steps + 1
+        nwb.nw_release_workspace()
+        del hs, hr
+    elif B > 1:
+        out["e2e"] = None
+    gpu_last = S[n].cpu().numpy() if B == 1 else None
+    if rank == 0 and not args.no_cpu:
+        out["cpu_baseline"] = cpu_baseline(cfg, gpu_last)
+    if rank == 0:
+        print(json.dumps(out), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

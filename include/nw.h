@@ -1,0 +1,178 @@
+/*
+ * nw.h — C-ABI of libnwb200.so: Needleman–Wunsch score-matrix fill on B200 (sm_100a).
+ *
+ * THE BOUNDARY of this repository.  Everything below the entry points runs in
+ * hand-written CUDA kernels (paper_conf_sc_munksgaardhso22_b200/csrc/); nothing here falls
+ * back to the CPU.  No torch types: plain pointers, sizes and an opaque stream handle.
+ *
+ * What is computed (PAPER.md = /root/reference/PAPER.md, cited P:<line>):
+ *   The paper's NW running example (Fig. 2) fills an int32 matrix
+ *   whose row 0 and column 0 are given (the Fig. 2 loops start at 1), using Rodinia's cell
+ *   function (BASELINE.json north_star; reading R1):
+ *
+ *       score[i][j] = max(score[i-1][j-1] + ref[i][j], score[i-1][j] - p, score[i][j-1] - p)
+ *                                                                  for 1 <= i, j <= n.
+ *
+ *   The blocked anti-diagonal wavefront and the short-circuited in-place update
+ *   (each tile's result written straight into its LMAD slice W of score, P:512-516,
+ *   P:616-656) are how the kernels compute it; the result is the unique matrix fixed by the
+ *   recurrence and the borders (reading R13), bit-identical to oracle/nw_ref.c.
+ *
+ * Conventions shared by every entry point
+ *   - Matrices are row-major int32 with a leading dimension (pitch, in ELEMENTS):
+ *     element (i, j) is at base[i * ld + j].  Default pitch is n + 1 (Rodinia layout).
+ *   - score: row 0 and column 0 are READ-ONLY inputs (borders); rows/cols 1..n are
+ *     WRITE-ONLY outputs — the interior is never read before it is written, so a call is
+ *     idempotent and may be re-run after a failure.  ref: rows/cols 1..n are read; row 0 /
+ *     column 0 are ignored.  ref must not overlap score.
+ *   - Device pointers are owned by the caller and must be 4-byte aligned.
+ *   - `stream` is a cudaStream_t (NULL = legacy default stream).  Work is ENQUEUED and the
+ *     call returns; results are visible after the caller synchronises the stream.
+ *   - `tile` b in {0, 16, 32, 64, 128} selects the width W of the tile-column band one warp
+ *     owns (W = 32K, K columns per lane): b in {16, 32, 64} -> W = 64 (K = 2; narrower b x b
+ *     tiles are processed 64/b side by side, because conflict-free shared staging needs an
+ *     even K), b in {0, 128} -> W = 128 (K = 4, the default).  The result does not depend
+ *     on it (reading R8).
+ *   - Any n >= 0 is accepted (ragged last band: n need not be a multiple of b).
+ *   - Validation is synchronous and happens before anything is enqueued.  Range contract:
+ *     0 <= penalty and 2*n*penalty + n*NW_REF_MAX < 2^31 (else NW_ERANGE), |ref| <= NW_REF_MAX
+ *     and |border| <= 2^30 are the caller's promise (int32 arithmetic cannot overflow then).
+ *   - Asynchronous device faults (including the spin watchdog's trap) surface
+ *     as CUDA errors at the caller's next synchronisation of the stream.
+ *   - No exception or abort crosses the ABI.  Entry points are thread-safe; internal
+ *     workspace (ticket counter + epoch-tagged border buffers) is cached per (device, stream)
+ *     and released by nw_release_workspace().
+ */
+#ifndef NWB200_NW_H
+#define NWB200_NW_H
+#include <stdint.h>
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define NW_REF_MAX 1024
+#define NW_ABI_VERSION 1
+
+typedef enum {
+  NW_OK = 0,
+  NW_EINVAL = 1, /* null pointer, negative size, bad tile, ld < n+1, overlap, misaligned   */
+  NW_ERANGE = 2, /* penalty < 0 or 2*n*p + n*NW_REF_MAX >= 2^31 (int32 could overflow)     */
+  NW_ECUDA = 3,  /* a CUDA runtime call failed (nw_last_cuda_error() has the code)          */
+  NW_ENOMEM = 4, /* workspace allocation failed                                             */
+  NW_ECOMM = 5   /* sharded call with inconsistent peer / halo description                  */
+} nw_status;
+
+const char* nw_status_str(int status);
+int nw_abi_version(void);
+int nw_last_cuda_error(void); /* cudaError_t of the last NW_ECUDA in this thread */
+
+/* ---- single pair -------------------------------------------------------------------
+ * Persistent wavefront kernel (DESIGN.md §4 "strip kernel"): one launch; warps claim
+ * tile-column bands in wavefront order through an atomic ticket; band k+1 consumes band k's
+ * right border column through epoch-tagged ready entries (ready flag fused with the value,
+ * P:636-645 / Fig. 9 ordering); every tile is written in place (short-circuited).
+ * score, ref: (n+1) x (n+1), pitch n+1. */
+nw_status nw_fill(int32_t* score, const int32_t* ref, int64_t n, int32_t penalty, int32_t tile,
+                  void* stream);
+
+/* Same with explicit pitches (elements): ld_score >= n+1, ld_ref >= n+1. */
+nw_status nw_fill_ld(int32_t* score, int64_t ld_score, const int32_t* ref, int64_t ld_ref,
+                     int64_t n, int32_t penalty, int32_t tile, void* stream);
+
+/* ---- batch of independent pairs (BASELINE.json config 4) ---------------------------
+ * score, ref: [batch][n+1][n+1] contiguous (pair stride (n+1)^2 elements).  One launch;
+ * tickets enumerate (pair, band) so pairs are independent and need no collective. */
+nw_status nw_fill_batch(int32_t* score, const int32_t* ref, int64_t batch, int64_t n,
+                        int32_t penalty, int32_t tile, void* stream);
+
+/* General strided batch: pair k's score at score + k*stride_score, pitch ld_score. */
+nw_status nw_fill_batch_ld(int32_t* score, int64_t ld_score, int64_t stride_score,
+                           const int32_t* ref, int64_t ld_ref, int64_t stride_ref, int64_t batch,
+                           int64_t n, int32_t penalty, int32_t tile, void* stream);
+
+/* ---- one pair split into column strips across GPUs (BASELINE.json config 5) -------
+ * SPMD: every rank calls this with its own strip.  Rank g owns global columns
+ * (col0, col0 + w]; its LOCAL matrices are (n+1) x (w+1) with pitch ld:
+ *   local score row 0 = global row 0 columns col0..col0+w (col 0 = the corner (0, col0));
+ *   local score column 0, rows >= 1: the global left border (read only when halo_in == NULL,
+ *   i.e. on rank 0); local ref column 0 unused.
+ * halo_in  : (n+1) uint64 entries on THIS device, written by rank g-1's kernel
+ *            (entry i = (epoch << 32) | (uint32) score[i][col0]); NULL on rank 0.
+ *            Must be zero-filled once before first use; never needs resetting after.
+ * halo_out : rank g+1's halo_in (a peer-mapped pointer, e.g. torch symmetric memory) or
+ *            NULL on the last rank.  Written with st.relaxed.sys, one entry per row as soon
+ *            as the row's last column is final — the NVLink border push is fused into the
+ *            wavefront kernel (no host involvement, no separate send/recv).
+ * epoch    : nonzero, identical on all ranks for one collective call, strictly increasing
+ *            across calls that reuse the same halo buffers.  The caller must not start call
+ *            e+1 on rank g+1... until every rank finished call e (one barrier per call). */
+typedef struct {
+  int32_t* score;
+  int64_t ld_score;
+  const int32_t* ref;
+  int64_t ld_ref;
+  int64_t n;   /* rows 1..n                                  */
+  int64_t w;   /* local interior columns 1..w                */
+  const uint64_t* halo_in;
+  uint64_t* halo_out;
+  uint32_t epoch;
+  int32_t halo_out_is_peer; /* 1: halo_out lives on another GPU (system-scope stores) */
+} nw_strip;
+
+nw_status nw_fill_sharded(const nw_strip* strip, int32_t penalty, int32_t tile, void* stream);
+
+/* ---- end to end from HOST memory (bench e2e) ---------------------------------------
+ * Copies ref (rows 1..n) and the borders host->device, runs nw_fill, copies the full score
+ * matrix device->host.  Host buffers: (n+1)x(n+1) int32, pitch n+1; pinned memory is
+ * fastest.  Synchronous: returns when score_host holds the result.  Device buffers are
+ * cached per device and freed by nw_release_workspace(). */
+nw_status nw_fill_host(int32_t* score_host, const int32_t* ref_host, int64_t n, int32_t penalty,
+                       int32_t tile, int32_t device);
+
+/* ---- the paper's / Rodinia's structure, kept as baselines ----------------------------
+ * nw_fill_diagonal: one kernel launch per tile anti-diagonal d = 0..2q-2 (q = ceil(n/b)),
+ *   one CTA per b x b tile, the tile staged in shared memory from its LMAD slices Rvert /
+ *   Rhoriz (generalised to both halves in DESIGN.md §5) and written back in
+ *   place into W (the "Opt." short-circuited form of P:503-521).  tile b in {16, 32, 64}.
+ * nw_fill_unopt: the same schedule WITHOUT short-circuiting (the paper's "Unopt."
+ *   column of Table I): each diagonal's tiles are written to a fresh temporary
+ *   X[#tiles][b][b] and a second kernel copies X into W (A[W] = X).
+ * Both: score/ref (n+1)x(n+1) with the given pitches; 2q-1 (resp. 2(2q-1)) launches. */
+nw_status nw_fill_diagonal(int32_t* score, int64_t ld_score, const int32_t* ref, int64_t ld_ref,
+                           int64_t n, int32_t penalty, int32_t tile, void* stream);
+nw_status nw_fill_unopt(int32_t* score, int64_t ld_score, const int32_t* ref, int64_t ld_ref,
+                        int64_t n, int32_t penalty, int32_t tile, void* stream);
+
+/* ---- introspection (host only; used by tests/test_schedule.py and the bench) ---------- */
+/* Band geometry the persistent kernel uses: band width W for `tile` (0 -> default). */
+int32_t nw_band_width(int32_t tile);
+/* Number of kernel launches one call of the given entry point enqueues (bench gpu_launches):
+ * kind 0 = nw_fill/_ld/_batch/_sharded, 1 = nw_fill_diagonal, 2 = nw_fill_unopt. */
+int64_t nw_launch_count(int32_t kind, int64_t n, int32_t tile);
+/* Paper Appendix-C LMADs of tile anti-diagonal d for the diagonal kernels (element offsets
+ * relative to element (0,0), pitch N): out[0..9] = {cnt, base, W.off, W.s0, W.s1, W.s2,
+ * Rvert.off, Rvert.s1, Rhoriz.off, Rhoriz.s1} with shapes W = (cnt:s0,b:s1,b:s2),
+ * Rvert = (cnt:s0, b+1:s1), Rhoriz = (cnt:s0, b:1).  Returns 0, or -1 for bad args. */
+int32_t nw_diag_lmad(int64_t n, int64_t N, int32_t tile, int64_t d, int64_t out[10]);
+/* The persistent kernel's schedule (the same __host__ __device__ helpers the kernel calls):
+ * at wavefront step `step` of band `band`, lane `lane` computes row out[0], columns
+ * out[1] .. out[1]+out[2]-1 (out[2] = 0: lane idle at this step).  Steps run 0 .. n+30;
+ * band b+1 consumes band b's last column row by row.  Returns 0, or -1 for bad args. */
+int32_t nw_strip_map(int64_t n, int64_t width, int32_t tile, int32_t band, int32_t step, int32_t lane,
+                     int64_t out[3]);
+/* Smem bytes / resident CTAs per SM of the strip kernel for `tile` on `device`. */
+nw_status nw_kernel_info(int32_t tile, int32_t device, int64_t* smem_bytes, int32_t* ctas_per_sm,
+                         int32_t* num_sms);
+
+/* Test hook: cap the persistent kernel's grid at `grid` CTAs (0 = automatic, #SMs x
+ * occupancy).  A 1-CTA grid must still finish (ticket order => deadlock freedom). */
+void nw_debug_set_grid(int32_t grid);
+
+/* Frees every cached workspace (device buffers, pinned staging).  Not thread-safe with
+ * concurrent nw_* calls. */
+void nw_release_workspace(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* NWB200_NW_H */

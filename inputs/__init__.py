@@ -174,3 +174,32 @@ def make_problem(n: int, p: int = 10, seed: int = SEED, family: str = "random", 
     if sentinel:
         fill_interior(score, SENTINEL)
     return score, ref
+
+
+def device_problem(n: int, p: int = 10, seed: int = SEED, device="cuda", score=None, ref=None,
+                   sentinel: bool = True, chunk_rows: int = 4096):
+    """The same Rodinia-style problem as make_problem(n, p, seed), built ON THE DEVICE (for the
+    large bench configs): sequences from the C splitmix64 generator, ref = B62[a_i][b_j] by a
+    table gather in row chunks, global-alignment borders.  Optionally fills preallocated
+    (n+1, >= n+1) int32 views `score` / `ref` (e.g. one pair of a batch)."""
+    import torch
+    a, b = gen_pair(n, seed)
+    table = torch.from_numpy(blosum62()).to(device=device, dtype=torch.int32)
+    ta = torch.from_numpy(a.astype(np.int64)).to(device)
+    tb = torch.from_numpy(b.astype(np.int64)).to(device)
+    if score is None:
+        score = torch.empty((n + 1, n + 1), dtype=torch.int32, device=device)
+    if ref is None:
+        ref = torch.empty((n + 1, n + 1), dtype=torch.int32, device=device)
+    ref[0, : n + 1] = 0
+    ref[:, 0] = 0
+    rows_b = table[:, tb]                       # (24, n): B62[x][b_j] for every residue x
+    for i0 in range(0, n, chunk_rows):
+        i1 = min(n, i0 + chunk_rows)
+        ref[1 + i0:1 + i1, 1:n + 1] = rows_b[ta[i0:i1]]
+    steps = torch.arange(n + 1, device=device, dtype=torch.int64) * (-p)
+    score[0, : n + 1] = steps.to(torch.int32)
+    score[:, 0] = steps.to(torch.int32)
+    if sentinel:
+        score[1:, 1:n + 1] = SENTINEL
+    return score, ref

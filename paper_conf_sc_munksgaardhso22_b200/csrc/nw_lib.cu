@@ -1,0 +1,473 @@
+// nw_lib.cu — host side of libnwb200.so: the C ABI declared in include/nw.h.
+//
+// Synchronous validation, a per-(device, stream) workspace cache (ticket counter, epoch-tagged
+// band-border buffer, Unopt temporary), and the launches.  Every compute step runs in the
+// kernels of nw_strip.cuh / nw_diag.cuh; there is no CPU fallback: without a usable CUDA
+// device the entry points return NW_ECUDA.
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <cstdlib>
+#include <map>
+#include <mutex>
+#include <utility>
+
+#include "nw.h"
+#include "nw_diag.cuh"
+#include "nw_strip.cuh"
+
+using namespace nwb200;
+
+namespace {
+
+thread_local int g_last_cuda = 0;
+
+nw_status cuda_fail(cudaError_t e) {
+  g_last_cuda = static_cast<int>(e);
+  (void)cudaGetLastError();  // clear a non-sticky launch error
+  return NW_ECUDA;
+}
+#define NW_CU(x)                                    \
+  do {                                              \
+    cudaError_t e_ = (x);                           \
+    if (e_ != cudaSuccess) return cuda_fail(e_);    \
+  } while (0)
+
+constexpr int64_t kMaxN = (int64_t{1} << 30) - 64;
+
+int tile_to_k(int32_t tile) {
+  switch (tile) {
+    case 0: return 4;
+    case 16:
+    case 32:
+    case 64: return 2;
+    case 128: return 4;
+    default: return 0;
+  }
+}
+
+bool aligned4(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 3) == 0; }
+
+bool overlaps(const void* a, int64_t abytes, const void* b, int64_t bbytes) {
+  const uintptr_t a0 = reinterpret_cast<uintptr_t>(a), b0 = reinterpret_cast<uintptr_t>(b);
+  return a0 < b0 + static_cast<uintptr_t>(bbytes) && b0 < a0 + static_cast<uintptr_t>(abytes);
+}
+
+// bytes spanned by an (n+1) x (n+1) matrix with pitch ld (first to last element)
+int64_t span_bytes(int64_t n, int64_t ld) { return 4 * (n * ld + n + 1); }
+
+nw_status check_range(int64_t n, int32_t p) {
+  if (p < 0) return NW_ERANGE;
+  const long double worst = 2.0L * static_cast<long double>(n) * p + static_cast<long double>(n) * NW_REF_MAX;
+  if (worst >= 2147483648.0L) return NW_ERANGE;
+  return NW_OK;
+}
+
+struct DevInfo {
+  bool init = false;
+  int sms = 0;
+  int occ2 = 0, occ4 = 0;
+};
+
+std::mutex g_mu;
+DevInfo g_dev[128];
+int g_debug_grid = 0;
+
+nw_status dev_info(int dev, DevInfo** out) {
+  if (dev < 0 || dev >= 128) return NW_EINVAL;
+  DevInfo& d = g_dev[dev];
+  if (!d.init) {
+    NW_CU(cudaDeviceGetAttribute(&d.sms, cudaDevAttrMultiProcessorCount, dev));
+    NW_CU(cudaFuncSetAttribute(nw_strip_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               static_cast<int>(StripGeom<2>::kSmem)));
+    NW_CU(cudaFuncSetAttribute(nw_strip_kernel<4>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               static_cast<int>(StripGeom<4>::kSmem)));
+    NW_CU(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ2, nw_strip_kernel<2>, 32, StripGeom<2>::kSmem));
+    NW_CU(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ4, nw_strip_kernel<4>, 32, StripGeom<4>::kSmem));
+    if (d.occ2 < 1 || d.occ4 < 1) return cuda_fail(cudaErrorInvalidConfiguration);
+    d.init = true;
+  }
+  *out = &d;
+  return NW_OK;
+}
+
+struct Workspace {
+  unsigned long long* d_ticket = nullptr;
+  unsigned long long ticket_next = 0;
+  unsigned int* d_err = nullptr;
+  uint64_t* xbuf = nullptr;
+  size_t xbuf_entries = 0;
+  uint32_t epoch = 0;
+  int32_t* xtmp = nullptr;  // Unopt temporary X
+  size_t xtmp_elems = 0;
+};
+std::map<std::pair<int, void*>, Workspace*> g_ws;
+
+nw_status get_ws(int dev, cudaStream_t st, Workspace** out) {
+  auto key = std::make_pair(dev, static_cast<void*>(st));
+  auto it = g_ws.find(key);
+  if (it != g_ws.end()) {
+    *out = it->second;
+    return NW_OK;
+  }
+  Workspace* w = new Workspace();
+  cudaError_t e = cudaMalloc(reinterpret_cast<void**>(&w->d_ticket), 64);
+  if (e == cudaSuccess) e = cudaMemsetAsync(w->d_ticket, 0, 64, st);
+  if (e != cudaSuccess) {
+    delete w;
+    return cuda_fail(e);
+  }
+  w->d_err = reinterpret_cast<unsigned int*>(w->d_ticket + 1);
+  g_ws[key] = w;
+  *out = w;
+  return NW_OK;
+}
+
+nw_status ensure_xbuf(Workspace* w, size_t entries, cudaStream_t st) {
+  if (entries <= w->xbuf_entries && w->epoch < 0xFFFFFFF0u) return NW_OK;
+  if (w->xbuf) NW_CU(cudaFreeAsync(w->xbuf, st));
+  w->xbuf = nullptr;
+  w->xbuf_entries = 0;
+  const size_t want = entries < 1024 ? 1024 : entries;
+  NW_CU(cudaMallocAsync(reinterpret_cast<void**>(&w->xbuf), want * sizeof(uint64_t), st));
+  NW_CU(cudaMemsetAsync(w->xbuf, 0, want * sizeof(uint64_t), st));  // tag 0 = never written
+  w->xbuf_entries = want;
+  w->epoch = 0;
+  return NW_OK;
+}
+
+unsigned long long spin_limit_ns() {
+  static unsigned long long v = [] {
+    const char* s = std::getenv("NW_SPIN_LIMIT_MS");
+    const unsigned long long ms = s ? std::strtoull(s, nullptr, 10) : 20000ull;
+    return (ms ? ms : 20000ull) * 1000000ull;
+  }();
+  return v;
+}
+
+// One launch of the persistent kernel over `pairs` x ceil(width/W) bands.
+nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* ref, int64_t ldr, int64_t psr,
+                       int64_t pairs, int64_t n, int64_t width, int32_t p, int32_t tile, const uint64_t* halo_in,
+                       uint64_t* halo_out, uint32_t halo_epoch, int32_t halo_out_sys, cudaStream_t st) {
+  const int K = tile_to_k(tile);
+  const int W = 32 * K;
+  if (pairs == 0 || n == 0 || width == 0) return NW_OK;
+  int dev = 0;
+  NW_CU(cudaGetDevice(&dev));
+  std::lock_guard<std::mutex> lk(g_mu);
+  DevInfo* di = nullptr;
+  nw_status s = dev_info(dev, &di);
+  if (s != NW_OK) return s;
+  Workspace* w = nullptr;
+  s = get_ws(dev, st, &w);
+  if (s != NW_OK) return s;
+  const int64_t nbands = (width + W - 1) / W;
+  const size_t entries = static_cast<size_t>(pairs) * static_cast<size_t>(nbands - 1) * static_cast<size_t>(n + 1);
+  s = ensure_xbuf(w, entries, st);
+  if (s != NW_OK) return s;
+  StripParams P{};
+  P.score = score;
+  P.lds = lds;
+  P.pss = pss;
+  P.ref = ref;
+  P.ldr = ldr;
+  P.psr = psr;
+  P.n = n;
+  P.width = width;
+  P.p = p;
+  P.nbands = static_cast<int32_t>(nbands);
+  P.ntasks = pairs * nbands;
+  P.xbuf = w->xbuf;
+  P.epoch = ++w->epoch;
+  P.halo_in = halo_in;
+  P.halo_out = halo_out;
+  P.halo_epoch = halo_epoch;
+  P.halo_out_sys = halo_out_sys;
+  P.ticket = w->d_ticket;
+  P.err = w->d_err;
+  P.spin_limit_ns = spin_limit_ns();
+  const int occ = K == 2 ? di->occ2 : di->occ4;
+  int64_t grid = static_cast<int64_t>(occ) * di->sms;
+  if (g_debug_grid > 0) grid = g_debug_grid;
+  if (grid > P.ntasks) grid = P.ntasks;
+  P.ticket_base = w->ticket_next;
+  w->ticket_next += static_cast<unsigned long long>(P.ntasks + grid);  // every CTA draws one extra ticket
+  if (K == 2)
+    nw_strip_kernel<2><<<static_cast<unsigned>(grid), 32, StripGeom<2>::kSmem, st>>>(P);
+  else
+    nw_strip_kernel<4><<<static_cast<unsigned>(grid), 32, StripGeom<4>::kSmem, st>>>(P);
+  NW_CU(cudaGetLastError());
+  return NW_OK;
+}
+
+nw_status validate_pair(const int32_t* score, int64_t lds, const int32_t* ref, int64_t ldr, int64_t n,
+                        int32_t p, int32_t tile) {
+  if (!score || !ref) return NW_EINVAL;
+  if (n < 0 || n > kMaxN) return NW_EINVAL;
+  if (tile_to_k(tile) == 0) return NW_EINVAL;
+  if (lds < n + 1 || ldr < n + 1) return NW_EINVAL;
+  if (!aligned4(score) || !aligned4(ref)) return NW_EINVAL;
+  if (overlaps(score, span_bytes(n, lds), ref, span_bytes(n, ldr))) return NW_EINVAL;
+  return check_range(n, p);
+}
+
+template <int B>
+nw_status run_diag(int32_t* score, int64_t lds, const int32_t* ref, int64_t ldr, int64_t n, int32_t p, bool unopt,
+                   cudaStream_t st) {
+  const int q = static_cast<int>((n + B - 1) / B);
+  int32_t* X = nullptr;
+  if (unopt) {
+    int dev = 0;
+    NW_CU(cudaGetDevice(&dev));
+    std::lock_guard<std::mutex> lk(g_mu);
+    Workspace* w = nullptr;
+    nw_status s = get_ws(dev, st, &w);
+    if (s != NW_OK) return s;
+    const size_t need = static_cast<size_t>(q) * B * B;
+    if (need > w->xtmp_elems) {
+      if (w->xtmp) NW_CU(cudaFreeAsync(w->xtmp, st));
+      w->xtmp = nullptr;
+      w->xtmp_elems = 0;
+      NW_CU(cudaMallocAsync(reinterpret_cast<void**>(&w->xtmp), need * sizeof(int32_t), st));
+      w->xtmp_elems = need;
+    }
+    X = w->xtmp;
+  }
+  for (int d = 0; d <= 2 * q - 2; ++d) {
+    const DiagLmad L = diag_lmad(q, B, lds, d);
+    nw_diag_kernel<B><<<static_cast<unsigned>(L.cnt), B, 0, st>>>(score, lds, ref, ldr, static_cast<int>(n), p, d,
+                                                                   q, X);
+    if (unopt) nw_diag_copy_kernel<B><<<static_cast<unsigned>(L.cnt), B, 0, st>>>(score, lds, static_cast<int>(n), d, q, X);
+  }
+  NW_CU(cudaGetLastError());
+  return NW_OK;
+}
+
+nw_status diag_entry(int32_t* score, int64_t lds, const int32_t* ref, int64_t ldr, int64_t n, int32_t p,
+                     int32_t tile, void* stream, bool unopt) {
+  if (tile != 16 && tile != 32 && tile != 64) return NW_EINVAL;
+  nw_status s = validate_pair(score, lds, ref, ldr, n, p, tile);
+  if (s != NW_OK || n == 0) return s;
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  switch (tile) {
+    case 16: return run_diag<16>(score, lds, ref, ldr, n, p, unopt, st);
+    case 32: return run_diag<32>(score, lds, ref, ldr, n, p, unopt, st);
+    default: return run_diag<64>(score, lds, ref, ldr, n, p, unopt, st);
+  }
+}
+
+struct HostBufs {
+  int32_t* score = nullptr;
+  int32_t* ref = nullptr;
+  size_t elems = 0;
+  cudaStream_t st = nullptr;
+};
+HostBufs g_host[128];
+
+}  // namespace
+
+extern "C" {
+
+const char* nw_status_str(int status) {
+  switch (status) {
+    case NW_OK: return "NW_OK";
+    case NW_EINVAL: return "NW_EINVAL: invalid argument (pointer, size, tile, pitch, alignment or overlap)";
+    case NW_ERANGE: return "NW_ERANGE: penalty < 0 or int32 could overflow (2*n*p + n*NW_REF_MAX >= 2^31)";
+    case NW_ECUDA: return "NW_ECUDA: a CUDA runtime call failed (see nw_last_cuda_error)";
+    case NW_ENOMEM: return "NW_ENOMEM: workspace allocation failed";
+    case NW_ECOMM: return "NW_ECOMM: inconsistent sharded strip / halo description";
+    default: return "NW_UNKNOWN";
+  }
+}
+
+int nw_abi_version(void) { return NW_ABI_VERSION; }
+int nw_last_cuda_error(void) { return g_last_cuda; }
+
+nw_status nw_fill_ld(int32_t* score, int64_t ld_score, const int32_t* ref, int64_t ld_ref, int64_t n,
+                     int32_t penalty, int32_t tile, void* stream) {
+  nw_status s = validate_pair(score, ld_score, ref, ld_ref, n, penalty, tile);
+  if (s != NW_OK || n == 0) return s;
+  return launch_strip(score, ld_score, 0, ref, ld_ref, 0, 1, n, n, penalty, tile, nullptr, nullptr, 0, 0,
+                      static_cast<cudaStream_t>(stream));
+}
+
+nw_status nw_fill(int32_t* score, const int32_t* ref, int64_t n, int32_t penalty, int32_t tile, void* stream) {
+  return nw_fill_ld(score, n + 1, ref, n + 1, n, penalty, tile, stream);
+}
+
+nw_status nw_fill_batch_ld(int32_t* score, int64_t ld_score, int64_t stride_score, const int32_t* ref,
+                           int64_t ld_ref, int64_t stride_ref, int64_t batch, int64_t n, int32_t penalty,
+                           int32_t tile, void* stream) {
+  if (batch < 0) return NW_EINVAL;
+  if (!score || !ref || n < 0 || n > kMaxN || tile_to_k(tile) == 0) return NW_EINVAL;
+  if (ld_score < n + 1 || ld_ref < n + 1) return NW_EINVAL;
+  if (!aligned4(score) || !aligned4(ref)) return NW_EINVAL;
+  const int64_t ss = span_bytes(n, ld_score) / 4, sr = span_bytes(n, ld_ref) / 4;
+  if (batch > 1 && (stride_score < ss || stride_ref < sr)) return NW_EINVAL;  // pairs must not overlap
+  if (batch > 0 && overlaps(score, 4 * ((batch - 1) * stride_score + ss), ref, 4 * ((batch - 1) * stride_ref + sr)))
+    return NW_EINVAL;
+  nw_status s = check_range(n, penalty);
+  if (s != NW_OK || batch == 0 || n == 0) return s;
+  return launch_strip(score, ld_score, stride_score, ref, ld_ref, stride_ref, batch, n, n, penalty, tile, nullptr,
+                      nullptr, 0, 0, static_cast<cudaStream_t>(stream));
+}
+
+nw_status nw_fill_batch(int32_t* score, const int32_t* ref, int64_t batch, int64_t n, int32_t penalty,
+                        int32_t tile, void* stream) {
+  const int64_t st = (n + 1) * (n + 1);
+  return nw_fill_batch_ld(score, n + 1, st, ref, n + 1, st, batch, n, penalty, tile, stream);
+}
+
+nw_status nw_fill_sharded(const nw_strip* sp, int32_t penalty, int32_t tile, void* stream) {
+  if (!sp) return NW_EINVAL;
+  const nw_strip& S = *sp;
+  if (!S.score || !S.ref || S.n < 0 || S.n > kMaxN || S.w < 0 || S.w > kMaxN) return NW_EINVAL;
+  if (tile_to_k(tile) == 0) return NW_EINVAL;
+  if (S.ld_score < S.w + 1 || S.ld_ref < S.w + 1) return NW_EINVAL;
+  if (!aligned4(S.score) || !aligned4(S.ref)) return NW_EINVAL;
+  if (overlaps(S.score, 4 * (S.n * S.ld_score + S.w + 1), S.ref, 4 * (S.n * S.ld_ref + S.w + 1))) return NW_EINVAL;
+  if ((S.halo_in || S.halo_out) && S.epoch == 0) return NW_ECOMM;
+  if ((S.halo_in && (reinterpret_cast<uintptr_t>(S.halo_in) & 7)) ||
+      (S.halo_out && (reinterpret_cast<uintptr_t>(S.halo_out) & 7)))
+    return NW_ECOMM;
+  nw_status s = check_range(S.n > S.w ? S.n : S.w, penalty);
+  if (s != NW_OK || S.n == 0 || S.w == 0) return s;
+  return launch_strip(S.score, S.ld_score, 0, S.ref, S.ld_ref, 0, 1, S.n, S.w, penalty, tile, S.halo_in,
+                      S.halo_out, S.epoch, S.halo_out_is_peer, static_cast<cudaStream_t>(stream));
+}
+
+nw_status nw_fill_host(int32_t* score_host, const int32_t* ref_host, int64_t n, int32_t penalty, int32_t tile,
+                       int32_t device) {
+  if (!score_host || !ref_host || n < 0 || n > kMaxN || tile_to_k(tile) == 0) return NW_EINVAL;
+  if (device < 0 || device >= 128) return NW_EINVAL;
+  nw_status s = check_range(n, penalty);
+  if (s != NW_OK || n == 0) return s;
+  NW_CU(cudaSetDevice(device));
+  HostBufs& hb = g_host[device];
+  const size_t elems = static_cast<size_t>(n + 1) * static_cast<size_t>(n + 1);
+  {
+    std::lock_guard<std::mutex> lk(g_mu);
+    if (!hb.st) NW_CU(cudaStreamCreateWithFlags(&hb.st, cudaStreamNonBlocking));
+    if (elems > hb.elems) {
+      if (hb.score) NW_CU(cudaFree(hb.score));
+      if (hb.ref) NW_CU(cudaFree(hb.ref));
+      hb.score = hb.ref = nullptr;
+      hb.elems = 0;
+      NW_CU(cudaMalloc(reinterpret_cast<void**>(&hb.score), elems * 4));
+      NW_CU(cudaMalloc(reinterpret_cast<void**>(&hb.ref), elems * 4));
+      hb.elems = elems;
+    }
+  }
+  const size_t pitch = static_cast<size_t>(n + 1) * 4;
+  NW_CU(cudaMemcpyAsync(hb.ref, ref_host, elems * 4, cudaMemcpyHostToDevice, hb.st));
+  NW_CU(cudaMemcpyAsync(hb.score, score_host, pitch, cudaMemcpyHostToDevice, hb.st));  // row 0
+  NW_CU(cudaMemcpy2DAsync(hb.score + (n + 1), pitch, score_host + (n + 1), pitch, 4, static_cast<size_t>(n),
+                          cudaMemcpyHostToDevice, hb.st));  // column 0, rows 1..n
+  s = launch_strip(hb.score, n + 1, 0, hb.ref, n + 1, 0, 1, n, n, penalty, tile, nullptr, nullptr, 0, 0, hb.st);
+  if (s != NW_OK) return s;
+  NW_CU(cudaMemcpyAsync(score_host, hb.score, elems * 4, cudaMemcpyDeviceToHost, hb.st));
+  NW_CU(cudaStreamSynchronize(hb.st));
+  return NW_OK;
+}
+
+nw_status nw_fill_diagonal(int32_t* score, int64_t ld_score, const int32_t* ref, int64_t ld_ref, int64_t n,
+                           int32_t penalty, int32_t tile, void* stream) {
+  return diag_entry(score, ld_score, ref, ld_ref, n, penalty, tile, stream, false);
+}
+
+nw_status nw_fill_unopt(int32_t* score, int64_t ld_score, const int32_t* ref, int64_t ld_ref, int64_t n,
+                        int32_t penalty, int32_t tile, void* stream) {
+  return diag_entry(score, ld_score, ref, ld_ref, n, penalty, tile, stream, true);
+}
+
+int32_t nw_band_width(int32_t tile) { return 32 * tile_to_k(tile); }
+
+int64_t nw_launch_count(int32_t kind, int64_t n, int32_t tile) {
+  if (n <= 0) return 0;
+  if (kind == 0) return tile_to_k(tile) ? 1 : -1;
+  if (tile != 16 && tile != 32 && tile != 64) return -1;
+  const int64_t q = (n + tile - 1) / tile;
+  if (kind == 1) return 2 * q - 1;
+  if (kind == 2) return 2 * (2 * q - 1);
+  return -1;
+}
+
+int32_t nw_diag_lmad(int64_t n, int64_t N, int32_t tile, int64_t d, int64_t out[10]) {
+  if (!out || n < 1 || tile < 1 || N < n + 1) return -1;
+  const int64_t q = (n + tile - 1) / tile;
+  if (d < 0 || d > 2 * q - 2) return -1;
+  const DiagLmad L = diag_lmad(q, tile, N, d);
+  out[0] = L.cnt;
+  out[1] = L.base;
+  out[2] = L.base + N + 1;  // W offset
+  out[3] = L.s0;
+  out[4] = N;
+  out[5] = 1;
+  out[6] = L.base;  // Rvert offset
+  out[7] = N;
+  out[8] = L.base + 1;  // Rhoriz offset
+  out[9] = 1;
+  return 0;
+}
+
+nw_status nw_kernel_info(int32_t tile, int32_t device, int64_t* smem_bytes, int32_t* ctas_per_sm,
+                         int32_t* num_sms) {
+  const int K = tile_to_k(tile);
+  if (!K) return NW_EINVAL;
+  if (smem_bytes) *smem_bytes = static_cast<int64_t>(K == 2 ? StripGeom<2>::kSmem : StripGeom<4>::kSmem);
+  if (!ctas_per_sm && !num_sms) return NW_OK;
+  NW_CU(cudaSetDevice(device));
+  std::lock_guard<std::mutex> lk(g_mu);
+  DevInfo* di = nullptr;
+  nw_status s = dev_info(device, &di);
+  if (s != NW_OK) return s;
+  if (ctas_per_sm) *ctas_per_sm = K == 2 ? di->occ2 : di->occ4;
+  if (num_sms) *num_sms = di->sms;
+  return NW_OK;
+}
+
+int32_t nw_strip_map(int64_t n, int64_t width, int32_t tile, int32_t band, int32_t step, int32_t lane,
+                     int64_t out[3]) {
+  const int K = tile_to_k(tile);
+  if (!out || !K || n < 0 || width < 1 || lane < 0 || lane > 31 || band < 0) return -1;
+  const int W = 32 * K;
+  if (static_cast<int64_t>(band) * W >= width) return -1;
+  const int c0 = band_c0(band, W), ws = band_ws(width, band, W);
+  const int r = lane_row(step, lane);
+  int nc = ws - lane * K;
+  nc = nc < 0 ? 0 : (nc > K ? K : nc);
+  if (r < 1 || r > n) nc = 0;
+  out[0] = r;
+  out[1] = c0 + lane * K;
+  out[2] = nc;
+  return 0;
+}
+
+void nw_debug_set_grid(int32_t grid) { g_debug_grid = grid > 0 ? grid : 0; }
+
+void nw_release_workspace(void) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  for (auto& kv : g_ws) {
+    Workspace* w = kv.second;
+    cudaSetDevice(kv.first.first);
+    cudaStreamSynchronize(static_cast<cudaStream_t>(kv.first.second));
+    if (w->xbuf) cudaFree(w->xbuf);
+    if (w->xtmp) cudaFree(w->xtmp);
+    if (w->d_ticket) cudaFree(w->d_ticket);
+    delete w;
+  }
+  g_ws.clear();
+  for (int d = 0; d < 128; ++d) {
+    HostBufs& hb = g_host[d];
+    if (hb.score || hb.ref || hb.st) {
+      cudaSetDevice(d);
+      if (hb.st) cudaStreamSynchronize(hb.st);
+      if (hb.score) cudaFree(hb.score);
+      if (hb.ref) cudaFree(hb.ref);
+      if (hb.st) cudaStreamDestroy(hb.st);
+      hb = HostBufs();
+    }
+  }
+}
+
+}  // extern "C"

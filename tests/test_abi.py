@@ -1,0 +1,126 @@
+"""The C-ABI boundary (include/nw.h) on the CPU host: the library loads, exports every symbol
+the header declares, and its synchronous validation returns the documented status codes
+before touching CUDA.  No compute call runs here (there is no GPU)."""
+import ctypes
+import os
+import re
+import subprocess
+
+import pytest
+
+import paper_conf_sc_munksgaardhso22_b200 as nwb
+from paper_conf_sc_munksgaardhso22_b200 import (NW_ECOMM, NW_ECUDA, NW_EINVAL, NW_ERANGE, NW_OK,
+                                                 NwStrip)
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+HEADER = os.path.join(ROOT, "include", "nw.h")
+
+
+@pytest.fixture(scope="module")
+def L():
+    nwb.build()
+    return nwb.lib()
+
+
+def declared_functions():
+    src = open(HEADER).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    names = re.findall(r"^\s*(?:const\s+)?[A-Za-z_][A-Za-z0-9_]*\s*\*?\s+\*?([a-z_][a-z0-9_]*)\s*\(", src, re.M)
+    return sorted(set(names))
+
+
+def test_header_declares_the_boundary():
+    names = declared_functions()
+    for must in ("nw_fill", "nw_fill_ld", "nw_fill_batch", "nw_fill_batch_ld", "nw_fill_sharded",
+                 "nw_fill_host", "nw_fill_diagonal", "nw_fill_unopt", "nw_status_str"):
+        assert must in names
+
+
+def test_library_exports_every_declared_symbol(L):
+    out = subprocess.run(["nm", "-D", "--defined-only", nwb.LIB_PATH], capture_output=True, text=True).stdout
+    exported = set(re.findall(r" T (\w+)$", out, re.M))
+    missing = [f for f in declared_functions() if f not in exported]
+    assert not missing, missing
+    for f in declared_functions():
+        assert hasattr(L, f)
+
+
+def test_library_is_sm100a_only():
+    out = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "--list-elf", nwb.LIB_PATH],
+                         capture_output=True, text=True).stdout
+    assert "sm_100a" in out
+    sass = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "-sass", nwb.LIB_PATH],
+                          capture_output=True, text=True).stdout
+    assert "UBLKCP" in sass          # cp.async.bulk staging (TMA bulk engine)
+    assert "VIADDMNMX" in sass       # DPX add+max cell update
+
+
+def test_status_strings(L):
+    assert nwb.nw_status_str(NW_OK) == "NW_OK"
+    for s in range(1, 6):
+        assert nwb.nw_status_str(s).startswith("NW_E")
+    assert L.nw_abi_version() == 1
+
+
+FAKE_S = 0x10000000
+FAKE_R = 0x80000000
+
+
+def fill_ld(L, s, lds, r, ldr, n, p, tile):
+    return L.nw_fill_ld(s, lds, r, ldr, n, p, tile, None)
+
+
+def test_validation_codes(L):
+    n = 64
+    assert fill_ld(L, None, n + 1, FAKE_R, n + 1, n, 10, 16) == NW_EINVAL          # null
+    assert fill_ld(L, FAKE_S, n + 1, None, n + 1, n, 10, 16) == NW_EINVAL
+    assert fill_ld(L, FAKE_S, n + 1, FAKE_R, n + 1, -1, 10, 16) == NW_EINVAL       # n < 0
+    assert fill_ld(L, FAKE_S, n + 1, FAKE_R, n + 1, n, 10, 24) == NW_EINVAL        # bad tile
+    assert fill_ld(L, FAKE_S, n, FAKE_R, n + 1, n, 10, 16) == NW_EINVAL            # ld < n+1
+    assert fill_ld(L, FAKE_S, n + 1, FAKE_R, n, n, 10, 16) == NW_EINVAL
+    assert fill_ld(L, FAKE_S + 2, n + 1, FAKE_R, n + 1, n, 10, 16) == NW_EINVAL    # misaligned
+    assert fill_ld(L, FAKE_S, n + 1, FAKE_S + 400, n + 1, n, 10, 16) == NW_EINVAL  # overlap
+    assert fill_ld(L, FAKE_S, n + 1, FAKE_R, n + 1, n, -1, 16) == NW_ERANGE        # p < 0
+    big = 1 << 20
+    assert fill_ld(L, FAKE_S, big + 1, FAKE_S + (1 << 45), big + 1, big, 1000, 0) == NW_ERANGE  # overflow risk
+    assert fill_ld(L, FAKE_S, n + 1, FAKE_R, n + 1, 0, 10, 16) == NW_OK            # n == 0: no work
+    assert L.nw_fill(None, FAKE_R, n, 10, 0, None) == NW_EINVAL
+
+
+def test_no_cpu_fallback(L):
+    # valid arguments but no GPU in this container: the library must fail, not compute on the host
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("GPU present")
+    assert fill_ld(L, FAKE_S, 65, FAKE_R, 65, 64, 10, 16) == NW_ECUDA
+    assert L.nw_last_cuda_error() != 0
+
+
+def test_batch_and_sharded_validation(L):
+    n = 32
+    st = (n + 1) * (n + 1)
+    assert L.nw_fill_batch_ld(FAKE_S, n + 1, st, FAKE_R, n + 1, st, -1, n, 10, 0, None) == NW_EINVAL
+    assert L.nw_fill_batch_ld(FAKE_S, n + 1, st - 1, FAKE_R, n + 1, st, 2, n, 10, 0, None) == NW_EINVAL
+    assert L.nw_fill_batch_ld(FAKE_S, n + 1, st, FAKE_R, n + 1, st, 0, n, 10, 0, None) == NW_OK
+    assert L.nw_fill_sharded(None, 10, 0, None) == NW_EINVAL
+    s = NwStrip(FAKE_S, 17, FAKE_R, 17, 64, 16, None, 0x20000000, 0, 1)
+    assert L.nw_fill_sharded(ctypes.byref(s), 10, 0, None) == NW_ECOMM            # halo without epoch
+    s = NwStrip(FAKE_S, 17, FAKE_R, 17, 64, 16, 0x30000004, None, 5, 0)
+    assert L.nw_fill_sharded(ctypes.byref(s), 10, 0, None) == NW_ECOMM            # misaligned halo
+    s = NwStrip(FAKE_S, 16, FAKE_R, 17, 64, 16, None, None, 0, 0)
+    assert L.nw_fill_sharded(ctypes.byref(s), 10, 0, None) == NW_EINVAL           # ld < w+1
+
+
+def test_host_entry_validation(L):
+    assert L.nw_fill_host(None, None, 8, 10, 0, 0) == NW_EINVAL
+    assert L.nw_fill_diagonal(FAKE_S, 65, FAKE_R, 65, 64, 10, 128, None) == NW_EINVAL  # diag: b <= 64
+
+
+def test_band_width_and_launch_counts():
+    assert nwb.nw_band_width(0) == 128 and nwb.nw_band_width(128) == 128
+    assert nwb.nw_band_width(16) == nwb.nw_band_width(32) == nwb.nw_band_width(64) == 64
+    assert nwb.nw_band_width(7) == 0
+    assert nwb.nw_launch_count(0, 32768, 0) == 1                     # one persistent launch
+    assert nwb.nw_launch_count(1, 32768, 16) == 2 * 2048 - 1         # Rodinia: one per diagonal
+    assert nwb.nw_launch_count(2, 32768, 16) == 2 * (2 * 2048 - 1)   # Unopt: + one copy each
+    assert nwb.nw_launch_count(1, 1000, 16) == 2 * 63 - 1            # ragged q = ceil(n/b)

@@ -1,0 +1,202 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle, element by element.
+
+The bar is BIT-EXACT on every cell (integer work): the recurrence plus the
+borders determine the matrix uniquely (reading R13), so any schedule must reproduce the
+oracle's int32 values exactly.  The interior is pre-filled with the sentinel 0x80000000, so an
+unwritten cell fails too.  Inputs come from the seeded generator in inputs/ (no arithmetic of
+the method there); expected values only ever come from oracle/.
+"""
+import numpy as np
+import pytest
+
+import inputs
+import oracle
+
+torch = pytest.importorskip("torch")
+import paper_conf_sc_munksgaardhso22_b200 as nwb  # noqa: E402
+
+pytestmark = pytest.mark.gpu
+
+
+def to_dev(a, ld=None, offset=0):
+    """(n+1, n+1) host matrix -> CUDA int32 view with pitch ld and a base shifted by `offset`
+    elements inside a larger allocation (exercises every 16-byte phase of the rows)."""
+    n1 = a.shape[0]
+    ld = a.shape[1] if ld is None else ld
+    buf = torch.full((offset + n1 * ld + 8,), -7, dtype=torch.int32, device="cuda")
+    view = buf[offset:offset + n1 * ld].view(n1, ld)
+    view[:, : a.shape[1]] = torch.from_numpy(np.ascontiguousarray(a)).cuda()
+    return view
+
+
+def expect(score, ref, p):
+    return oracle.nw_ref(score.copy(), ref, p)
+
+
+def gpu_fill(score, ref, p, tile, fn=None, ld=None, offset=0):
+    n = score.shape[0] - 1
+    s = to_dev(score, ld, offset)
+    r = to_dev(ref, ld, (offset * 3) % 4)
+    (fn or nwb.nw_fill)(s, r, p, tile)
+    torch.cuda.synchronize()
+    return s[:, : n + 1].cpu().numpy()
+
+
+SIZES = [1, 2, 3, 15, 16, 17, 31, 32, 33, 63, 64, 65, 100, 127, 128, 129, 255, 256, 257, 1000, 1024]
+
+
+@pytest.mark.parametrize("tile", [0, 16, 64, 128])
+@pytest.mark.parametrize("n", SIZES)
+def test_fill_sizes(n, tile):
+    score, ref = inputs.make_problem(n, 10, seed=n)
+    np.testing.assert_array_equal(gpu_fill(score, ref, 10, tile), expect(score, ref, 10))
+
+
+@pytest.mark.parametrize("p", [0, 1, 3, 10, 1000])
+@pytest.mark.parametrize("family", ["random", "homologous", "const", "borders"])
+def test_fill_families(family, p):
+    n = 700
+    kw = {"family": "const", "const_ref": 5} if family == "const" else {"family": family}
+    if family == "borders":
+        kw = {"family": "random", "border_seed": 99}
+    score, ref = inputs.make_problem(n, p, seed=3, **kw)
+    for tile in (0, 32):
+        np.testing.assert_array_equal(gpu_fill(score, ref, p, tile), expect(score, ref, p))
+
+
+@pytest.mark.parametrize("ld_extra,offset", [(0, 1), (0, 2), (0, 3), (3, 0), (4, 0), (7, 1), (31, 2)])
+def test_fill_pitch_and_alignment(ld_extra, offset):
+    n = 517
+    score, ref = inputs.make_problem(n, 10, seed=11)
+    got = gpu_fill(score, ref, 10, 0, ld=n + 1 + ld_extra, offset=offset)
+    np.testing.assert_array_equal(got, expect(score, ref, 10))
+
+
+def test_config1_bit_exact_and_idempotent():
+    """BASELINE.json config 1: n=1024, p=10, tile=16, repeated back to back (Table I ran 1000x)."""
+    n, p = 1024, 10
+    score, ref = inputs.make_problem(n, p)
+    want = expect(score, ref, p)
+    s, r = to_dev(score), to_dev(ref)
+    for _ in range(200):
+        nwb.nw_fill(s, r, p, 16)
+    torch.cuda.synchronize()
+    np.testing.assert_array_equal(s.cpu().numpy(), want)
+
+
+@pytest.mark.parametrize("grid", [1, 3])
+def test_small_grids_deadlock_free(grid):
+    """Ticket order => a CTA only waits on bands held by running CTAs: a 1-CTA grid must finish."""
+    n = 600
+    score, ref = inputs.make_problem(n, 10, seed=5)
+    try:
+        nwb.nw_debug_set_grid(grid)
+        got = gpu_fill(score, ref, 10, 16)
+    finally:
+        nwb.nw_debug_set_grid(0)
+    np.testing.assert_array_equal(got, expect(score, ref, 10))
+
+
+def test_workspace_reuse_across_sizes():
+    """Epoch tags keep stale band borders of earlier calls (other n, other tile) harmless."""
+    for n, tile in [(300, 0), (1000, 64), (129, 0), (2000, 16), (300, 0)]:
+        score, ref = inputs.make_problem(n, 10, seed=n + tile)
+        np.testing.assert_array_equal(gpu_fill(score, ref, 10, tile), expect(score, ref, 10))
+
+
+@pytest.mark.parametrize("tile", [16, 32, 64])
+@pytest.mark.parametrize("n", [1, 16, 47, 64, 200, 1024])
+def test_diagonal_and_unopt(n, tile):
+    score, ref = inputs.make_problem(n, 10, seed=7 + n)
+    want = expect(score, ref, 10)
+    np.testing.assert_array_equal(gpu_fill(score, ref, 10, tile, fn=nwb.nw_fill_diagonal), want)
+    np.testing.assert_array_equal(gpu_fill(score, ref, 10, tile, fn=nwb.nw_fill_unopt), want)
+
+
+def test_fill_host_e2e():
+    n = 999
+    score, ref = inputs.make_problem(n, 10, seed=21)
+    want = expect(score, ref, 10)
+    got = score.copy()
+    nwb.nw_fill_host(got, ref, 10, 0, 0)
+    np.testing.assert_array_equal(got, want)
+
+
+@pytest.mark.parametrize("B,n,tile", [(1, 64, 0), (5, 100, 16), (7, 257, 0), (33, 64, 64), (3, 2048, 0)])
+def test_batch(B, n, tile):
+    probs = [inputs.make_problem(n, 10, seed=inputs.pair_seed(k)) for k in range(B)]
+    S = torch.from_numpy(np.stack([s for s, _ in probs])).cuda()
+    R = torch.from_numpy(np.stack([r for _, r in probs])).cuda()
+    nwb.nw_fill_batch(S, R, 10, tile)
+    torch.cuda.synchronize()
+    got = S.cpu().numpy()
+    for k, (s, r) in enumerate(probs):
+        np.testing.assert_array_equal(got[k], expect(s, r, 10), err_msg=f"pair {k}")
+
+
+def split_strips(score, ref, G):
+    """Cut a global problem into G column strips (local (n+1) x (w+1) matrices, col 0 = halo)."""
+    n = score.shape[0] - 1
+    bounds = [round(g * n / G) for g in range(G + 1)]
+    out = []
+    for g in range(G):
+        a, b = bounds[g], bounds[g + 1]
+        ls = score[:, a:b + 1].copy()
+        lr = ref[:, a:b + 1].copy()
+        if g > 0:
+            ls[1:, 0] = inputs.SENTINEL  # the halo must come from the left rank, not from here
+        out.append((a, b, ls, lr))
+    return out
+
+
+@pytest.mark.parametrize("G,n,tile", [(2, 256, 0), (3, 500, 16), (4, 1024, 0), (8, 1000, 64)])
+def test_sharded_single_device(G, n, tile):
+    """Config 5's protocol on one GPU: G strips launched in rank order on one stream, each
+    pushing its right border into the next strip's halo (epoch-tagged entries)."""
+    score, ref = inputs.make_problem(n, 10, seed=17)
+    want = expect(score, ref, 10)
+    strips = split_strips(score, ref, G)
+    halos = [torch.zeros(n + 1, dtype=torch.int64, device="cuda") for _ in range(G + 1)]
+    for epoch in (1, 2, 7):                        # re-use of halo buffers across calls
+        locs = []
+        for g, (a, b, ls, lr) in enumerate(strips):
+            s_dev, r_dev = to_dev(ls), to_dev(lr)
+            nwb.nw_fill_sharded(s_dev, r_dev, 10, halo_in=halos[g] if g > 0 else None,
+                                halo_out=halos[g + 1] if g < G - 1 else None, epoch=epoch, tile=tile)
+            locs.append(s_dev)
+        torch.cuda.synchronize()
+        for g, (a, b, ls, lr) in enumerate(strips):
+            got = locs[g].cpu().numpy()
+            np.testing.assert_array_equal(got[:, 1:], want[:, a + 1:b + 1], err_msg=f"strip {g} epoch {epoch}")
+        # halo entries carry the tag and the left neighbour's last column
+        h = halos[1].cpu().numpy().view(np.uint64)
+        assert (h[1:] >> np.uint64(32) == epoch).all()
+        np.testing.assert_array_equal((h[1:] & np.uint64(0xFFFFFFFF)).astype(np.uint32).view(np.int32),
+                                      want[1:, strips[0][1]])
+
+
+def _stream_compare(s_dev, score_row0, ref, n, p, chunk=2048):
+    """Full-size check with the O(n)-memory streaming oracle, rows in chunks."""
+    st = oracle.NwRefStream(n, p, score_row0)
+    for i0 in range(1, n + 1, chunk):
+        i1 = min(n + 1, i0 + chunk)
+        got = s_dev[i0:i1].cpu().numpy()
+        want = st.rows(ref[i0:i1], got[:, 0].copy())
+        np.testing.assert_array_equal(got, want, err_msg=f"rows {i0}..{i1}")
+    st.close()
+
+
+@pytest.mark.parametrize("n,tile", [(16384, 64), (32768, 0)])
+def test_full_size_configs_bit_exact(n, tile):
+    """BASELINE.json configs 2/3 at full size, in the launch configuration bench.py times:
+    every cell against the streaming oracle."""
+    p = 10
+    a, b = inputs.gen_pair(n, inputs.SEED)
+    ref = inputs.build_ref(a, b)
+    score = inputs.init_borders(inputs.aligned_matrix(n), p)
+    s_dev, r_dev = torch.from_numpy(score).cuda(), torch.from_numpy(ref).cuda()
+    s_dev[1:, 1:] = inputs.SENTINEL
+    nwb.nw_fill(s_dev, r_dev, p, tile)
+    nwb.nw_fill(s_dev, r_dev, p, tile)
+    torch.cuda.synchronize()
+    _stream_compare(s_dev, score[0], ref, n, p)
