@@ -59,3 +59,13 @@ def test_borders():
     s = inputs.init_borders(inputs.aligned_matrix(5, ld=9), 10)
     assert list(s[0, :6]) == [0, -10, -20, -30, -40, -50]
     assert list(s[:, 0]) == [0, -10, -20, -30, -40, -50]
+
+
+def test_device_problem_matches_host_builder():
+    """The device-side recipe (used by bench.py for the big configs) builds the same problem."""
+    import torch
+    for n, seed in [(1, 7), (50, 3), (129, 11)]:
+        s, r = inputs.make_problem(n, 10, seed=seed)
+        ds, dr = inputs.device_problem(n, 10, seed=seed, device="cpu", chunk_rows=17)
+        np.testing.assert_array_equal(ds.numpy(), s)
+        np.testing.assert_array_equal(dr.numpy(), r)
