@@ -186,6 +186,9 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--variant", default="strip", choices=["strip", "diagonal", "unopt"],
+                    help="ablation: the paper's per-diagonal structure (Opt) / Unopt instead of the "
+                         "persistent kernel")
     args = ap.parse_args()
     world = env_int("WORLD_SIZE", 1)
     rank = env_int("RANK", 0)
@@ -225,9 +228,16 @@ def main():
         cells_local = nb * n * n
     else:
         S, R = inputs.device_problem(n, p, device=dev)
+        if args.variant == "strip":
+            def step():
+                nwb.nw_fill(S, R, p, tile)
+        else:
+            if tile not in (16, 32, 64):
+                tile = cfg["tile"] = 16
+            fn = nwb.nw_fill_diagonal if args.variant == "diagonal" else nwb.nw_fill_unopt
 
-        def step():
-            nwb.nw_fill(S, R, p, tile)
+            def step():
+                fn(S, R, p, tile)
         cells_local = n * n
     torch.cuda.synchronize()
     stream = torch.cuda.current_stream()
@@ -259,13 +269,14 @@ def main():
     ms_per_step = total_ms / args.steps
     value = cells_total / (ms_per_step * 1e-3) / 1e9
     # roofline of the (only) kernel: 8 algorithmic bytes per interior cell (ref read + score write)
-    kern_ms = statistics.mean(per_launch)
+    kern_ms = statistics.mean(per_launch)   # == the step: one launch per step for the strip kernel
     achieved = 8.0 * cells_local / (kern_ms * 1e-3) / 1e9
     peak, peak_src = measured_peaks()
     roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
             "traffic": ncu_traffic(cfg["workload"], tile), "peak_source": peak_src,
             "algorithmic_bytes_per_launch": 8 * cells_local,
-            "kernel": "nw_strip_kernel<%d>" % (4 if tile in (0, 128) else 2),
+            "kernel": ("nw_strip_kernel<%d>" % (4 if tile in (0, 128) else 2)) if args.variant == "strip"
+            else f"nw_diag_kernel<{tile}> x{nwb.nw_launch_count(1, n, tile)} launches (+copies: unopt)",
             "kernel_ms_mean": kern_ms, "kernel_ms_median": statistics.median(per_launch)}
     out = {"metric": METRIC, "value": value, "unit": "GCUPS", "n_gpus": world, "steps": args.steps,
            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
@@ -275,7 +286,9 @@ def main():
                       "band_width": nwb.nw_band_width(tile), "pairs_per_rank": B // world if B > 1 else 1,
                       "l2": "inputs %.1f GB >> 126 MB L2 (no flush needed)" % (8.0 * (n + 1) ** 2 * B / 1e9),
                       "parallelism": f"dp{world}" if world > 1 else "single"},
-           "roofline": roof, "gpu_launches": args.steps * nwb.nw_launch_count(0, n, tile),
+           "roofline": roof,
+           "gpu_launches": args.steps * nwb.nw_launch_count({"strip": 0, "diagonal": 1, "unopt": 2}[args.variant], n, tile),
+           "variant": args.variant,
            "clocks": clk.summary()}
     # ---- e2e through the public C ABI with host buffers (H2D + kernel + D2H inside the timing)
     if B == 1 and args.e2e_steps > 0:

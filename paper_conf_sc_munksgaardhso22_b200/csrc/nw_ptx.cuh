@@ -80,6 +80,15 @@ __device__ __forceinline__ void st_relaxed_gpu(uint64_t* p, uint64_t v) {
 __device__ __forceinline__ void st_relaxed_sys(uint64_t* p, uint64_t v) {
   asm volatile("st.relaxed.sys.global.b64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
+// (lo, hi) as one 64-bit single-copy-atomic store: the epoch-tagged border entry {value, epoch}
+__device__ __forceinline__ void st_relaxed_gpu_v2(uint64_t* p, uint32_t lo, uint32_t hi) {
+  asm volatile("{ .reg .b64 e; mov.b64 e, {%1, %2}; st.relaxed.gpu.global.b64 [%0], e; }" ::"l"(p), "r"(lo), "r"(hi)
+               : "memory");
+}
+__device__ __forceinline__ void st_relaxed_sys_v2(uint64_t* p, uint32_t lo, uint32_t hi) {
+  asm volatile("{ .reg .b64 e; mov.b64 e, {%1, %2}; st.relaxed.sys.global.b64 [%0], e; }" ::"l"(p), "r"(lo), "r"(hi)
+               : "memory");
+}
 __device__ __forceinline__ uint64_t globaltimer_ns() {
   uint64_t t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));

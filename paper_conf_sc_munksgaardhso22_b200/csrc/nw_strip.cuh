@@ -36,6 +36,7 @@
 //     as a CUDA error instead of a hung GPU.
 #pragma once
 #include <cstdint>
+#include <type_traits>
 
 #include "nw_ptx.cuh"
 
@@ -91,7 +92,7 @@ struct StripParams {
 };
 
 template <int K>
-__global__ void __launch_bounds__(32) nw_strip_kernel(const StripParams P) {
+__global__ void __launch_bounds__(32, 1) nw_strip_kernel(const StripParams P) {
   using G = StripGeom<K>;
   constexpr int RS = G::RS;
   constexpr unsigned FULL = 0xffffffffu;
@@ -111,7 +112,6 @@ __global__ void __launch_bounds__(32) nw_strip_kernel(const StripParams P) {
   const int nch = (n + kCH - 1) / kCH;
   const int nsteps = n + 31;
   const int p = P.p;
-  const int ldr4 = static_cast<int>(P.ldr & 3), lds4 = static_cast<int>(P.lds & 3);
   int seq10 = 0;  // ref-chunk sequence number mod 10 (ring slot + mbarrier parity), kept across tasks
 
   for (;;) {
@@ -154,9 +154,14 @@ __global__ void __launch_bounds__(32) nw_strip_kernel(const StripParams P) {
     }
     const int32_t* const colp = S + (c0 - 1);  // plain left border column (band 0 without halo)
     const int out_lane = (ws - 1) / K, out_m = (ws - 1) % K;
-    const int baseR = static_cast<int>(((reinterpret_cast<uintptr_t>(R) >> 2) + c0) & 3);
-    const int baseS = static_cast<int>(((reinterpret_cast<uintptr_t>(S) >> 2) + c0) & 3);
     const int ref_row_base = (seq10 % kRefSlots) * kCH;
+    // Row slots are swizzled by the row's own global word address: element x of row r sits at
+    // slot(r) + (G(r) & 31) + x, G(r) = word address of (r, c0).  The 16-byte phase G & 3 keeps
+    // smem and global 16-byte alignment identical (bulk copies), and for an odd pitch the
+    // 32 skewed rows a warp touches hit 32 different banks.
+    const uintptr_t GR0 = (reinterpret_cast<uintptr_t>(R) >> 2) + c0;  // word address of (0, c0)
+    const uintptr_t GS0 = (reinterpret_cast<uintptr_t>(S) >> 2) + c0;
+    const int ldr32 = static_cast<int>(P.ldr & 31), lds32 = static_cast<int>(P.lds & 31);
 
     auto load_border = [&](int row) -> uint64_t {
       if (row > n) return 0ull;
@@ -178,14 +183,15 @@ __global__ void __launch_bounds__(32) nw_strip_kernel(const StripParams P) {
         // never read past the matrix end: the final row of the last band loads its tail scalar
         const bool tail_scalar = (r == n) && last_band;
         const uintptr_t e0 = tail_scalar ? (ge & ~static_cast<uintptr_t>(15)) : ((ge + 15) & ~static_cast<uintptr_t>(15));
-        int32_t* drow = ref_ring + ((ref_row_base + r - 1) % kRefRows) * RS + (((r >> 2) & 7) << 2);
+        const int gw = static_cast<int>((gs >> 2) & 31);
+        int32_t* drow = ref_ring + ((ref_row_base + r - 1) % kRefRows) * RS + (gw & ~3);
         if (e0 > s0) {
           bytes = static_cast<uint32_t>(e0 - s0);
           src = reinterpret_cast<const void*>(s0);
           dst = smem_u32(drow);
         }
         if (tail_scalar) {
-          const int a = static_cast<int>((gs >> 2) & 3);
+          const int a = gw & 3;
           for (int x = e0 > gs ? static_cast<int>((e0 - gs) >> 2) : 0; x < ws; ++x) drow[a + x] = __ldg(g + x);
         }
       }
@@ -201,8 +207,7 @@ __global__ void __launch_bounds__(32) nw_strip_kernel(const StripParams P) {
       int32_t* g = S + static_cast<long long>(r) * P.lds + c0;
       const uintptr_t gs = reinterpret_cast<uintptr_t>(g), ge = gs + 4u * ws;
       const uintptr_t as = (gs + 15) & ~static_cast<uintptr_t>(15), ae = ge & ~static_cast<uintptr_t>(15);
-      const int32_t* srow =
-          sc_ring + ((r - 1) & (kScRows - 1)) * RS + (((r >> 2) & 7) << 2) + static_cast<int>((gs >> 2) & 3);
+      const int32_t* srow = sc_ring + ((r - 1) & (kScRows - 1)) * RS + static_cast<int>((gs >> 2) & 31);
       if (t < kCH) {
         if (ae > as) bulk_s2g(reinterpret_cast<void*>(as), smem_u32(srow) + static_cast<uint32_t>(as - gs),
                               static_cast<uint32_t>(ae - as));
@@ -221,10 +226,98 @@ __global__ void __launch_bounds__(32) nw_strip_kernel(const StripParams P) {
     int Lprev = (t * K < ws) ? __ldg(S + c0 + t * K - 1) : 0;  // diag input of the first row
     int vlast = Pv[K - 1];
     uint64_t cur = load_border(1 + t), nxt = load_border(33 + t);
+    int win_base = 1;  // cur holds border rows win_base + t
+    // true when every row of the window is published (or beyond n): no per-step tag checks
+    auto window_valid = [&]() -> bool {
+      if (lin == nullptr) return true;
+      return __all_sync(FULL, static_cast<uint32_t>(cur >> 32) == lin_epoch || win_base + t > n) != 0;
+    };
+    bool wvalid = window_valid();
+    // per-lane incremental addressing for row r = step + 1 - t (starts at r0 = 1 - t)
+    const int r0 = 1 - t;
+    int ref_off = (((ref_row_base + r0 - 1) % kRefRows + kRefRows) % kRefRows) * RS;
+    int sc_off = ((r0 - 1) & (kScRows - 1)) * RS;
+    int gR = static_cast<int>((GR0 + static_cast<uintptr_t>(static_cast<intptr_t>(r0) * P.ldr)) & 31);
+    int gS = static_cast<int>((GS0 + static_cast<uintptr_t>(static_cast<intptr_t>(r0) * P.lds)) & 31);
+    uint64_t* lout_row = lout != nullptr ? lout + r0 : nullptr;
+    const bool do_out = lout != nullptr && t == out_lane;
+    const bool out_full = out_m == K - 1;
     fence_proxy_async();
     __syncwarp();
     if (0 < nch) issue_ref(0);
     if (1 < nch) issue_ref(1);
+
+    // one wavefront step; ALL = every lane's row is in 1..n (steady state, no predicates)
+    auto step = [&](const int sig, auto all_tag) {
+      constexpr bool ALL = decltype(all_tag)::value;
+      const int from_left = __shfl_up_sync(FULL, vlast, 1);
+      const int idx = sig & 31;
+      int bval = __shfl_sync(FULL, static_cast<int>(static_cast<uint32_t>(cur)), idx);
+      if (!wvalid) {
+        uint32_t bep = __shfl_sync(FULL, static_cast<uint32_t>(cur >> 32), idx);
+        if (bep != lin_epoch && sig < n) {  // left band has not published row sig+1 yet
+          const int rowb = win_base + t;
+          const uint64_t t0 = globaltimer_ns();
+          for (;;) {
+            cur = load_border(rowb);
+            bep = __shfl_sync(FULL, static_cast<uint32_t>(cur >> 32), idx);
+            if (bep == lin_epoch) break;
+            if (globaltimer_ns() - t0 > P.spin_limit_ns) {
+              if (t == 0) atomicExch(P.err, kErrWatchdog);
+              __trap();
+            }
+          }
+          bval = __shfl_sync(FULL, static_cast<int>(static_cast<uint32_t>(cur)), idx);
+          wvalid = window_valid();
+        }
+      }
+      const int L = (t == 0) ? bval : from_left;
+      bool active = true;
+      if (!ALL) {
+        const int r = lane_row(sig, t);
+        active = r >= 1 && r <= n;
+      }
+      if (active) {
+        const int32_t* rrow = ref_ring + ref_off + gR + t * K;
+        int32_t* srow = sc_ring + sc_off + gS + t * K;
+        int rv[K];
+#pragma unroll
+        for (int m = 0; m < K; ++m) rv[m] = rrow[m];
+        int d = Lprev, l = L;
+#pragma unroll
+        for (int m = 0; m < K; ++m) {
+          const int x = __viaddmax_s32(Pv[m], -p, d + rv[m]);  // max(up - p, diag + ref)
+          const int v = __viaddmax_s32(l, -p, x);              // max(left - p, .)
+          d = Pv[m];
+          Pv[m] = v;
+          l = v;
+        }
+        Lprev = L;
+#pragma unroll
+        for (int m = 0; m < K; ++m) srow[m] = Pv[m];
+        if (do_out) {
+          int vo = Pv[K - 1];
+          if (!out_full) {
+#pragma unroll
+            for (int m = 0; m < K - 1; ++m)
+              if (m == out_m) vo = Pv[m];
+          }
+          if (lout_sys)
+            st_relaxed_sys_v2(lout_row, static_cast<uint32_t>(vo), lout_epoch);
+          else
+            st_relaxed_gpu_v2(lout_row, static_cast<uint32_t>(vo), lout_epoch);
+        }
+      }
+      vlast = Pv[K - 1];
+      // advance this lane to row r+1
+      ref_off += RS;
+      if (ref_off >= kRefRows * RS) ref_off -= kRefRows * RS;
+      sc_off += RS;
+      if (sc_off >= kScRows * RS) sc_off -= kScRows * RS;
+      gR = (gR + ldr32) & 31;
+      gS = (gS + lds32) & 31;
+      ++lout_row;
+    };
 
     for (int Q = 0; Q <= nch + 2; ++Q) {
       const int sig0 = Q * kCH;
@@ -246,68 +339,20 @@ __global__ void __launch_bounds__(32) nw_strip_kernel(const StripParams P) {
       if (sig0 >= nsteps) continue;
       if ((sig0 & 31) == 0 && sig0 > 0) {
         cur = nxt;
+        win_base = sig0 + 1;
         nxt = load_border(sig0 + 33 + t);
+        wvalid = window_valid();
       }
       // ---- 16 wavefront steps: lane t computes row sig+1-t, columns c0+tK .. c0+tK+K-1
-#pragma unroll 2
-      for (int j = 0; j < kCH; ++j) {
-        const int sig = sig0 + j;
-        if (sig >= nsteps) break;
-        const int r = lane_row(sig, t);
-        const int from_left = __shfl_up_sync(FULL, vlast, 1);
-        const int idx = sig & 31;
-        int bval = __shfl_sync(FULL, static_cast<int>(static_cast<uint32_t>(cur)), idx);
-        if (lin != nullptr) {
-          uint32_t bep = __shfl_sync(FULL, static_cast<uint32_t>(cur >> 32), idx);
-          if (bep != lin_epoch && sig < n) {  // left band has not published row sig+1 yet
-            const int rowb = sig - idx + 1 + t;
-            const uint64_t t0 = globaltimer_ns();
-            for (;;) {
-              cur = load_border(rowb);
-              bep = __shfl_sync(FULL, static_cast<uint32_t>(cur >> 32), idx);
-              if (bep == lin_epoch) break;
-              if (globaltimer_ns() - t0 > P.spin_limit_ns) {
-                if (t == 0) atomicExch(P.err, kErrWatchdog);
-                __trap();
-              }
-            }
-            bval = __shfl_sync(FULL, static_cast<int>(static_cast<uint32_t>(cur)), idx);
-          }
+      if (sig0 >= 31 && sig0 + kCH <= n) {  // steady state: all 32 lanes on rows 1..n
+#pragma unroll
+        for (int j = 0; j < kCH; ++j) step(sig0 + j, std::true_type{});
+      } else {
+#pragma unroll 1
+        for (int j = 0; j < kCH; ++j) {
+          if (sig0 + j >= nsteps) break;
+          step(sig0 + j, std::false_type{});
         }
-        const int L = (t == 0) ? bval : from_left;
-        if (r >= 1 && r <= n) {
-          const int swz = ((r >> 2) & 7) << 2;
-          const int32_t* rrow = ref_ring + ((ref_row_base + r - 1) % kRefRows) * RS + swz +
-                                ((baseR + (r & 3) * ldr4) & 3) + t * K;
-          int32_t* srow = sc_ring + ((r - 1) & (kScRows - 1)) * RS + swz + ((baseS + (r & 3) * lds4) & 3) + t * K;
-          int rv[K];
-#pragma unroll
-          for (int m = 0; m < K; ++m) rv[m] = rrow[m];
-          int d = Lprev, l = L;
-#pragma unroll
-          for (int m = 0; m < K; ++m) {
-            const int x = __viaddmax_s32(Pv[m], -p, d + rv[m]);  // max(up - p, diag + ref)
-            const int v = __viaddmax_s32(l, -p, x);              // max(left - p, .)
-            d = Pv[m];
-            Pv[m] = v;
-            l = v;
-          }
-          Lprev = L;
-#pragma unroll
-          for (int m = 0; m < K; ++m) srow[m] = Pv[m];
-          if (lout != nullptr && t == out_lane) {
-            int vo = Pv[K - 1];
-#pragma unroll
-            for (int m = 0; m < K - 1; ++m)
-              if (m == out_m) vo = Pv[m];
-            const uint64_t e = (static_cast<uint64_t>(lout_epoch) << 32) | static_cast<uint32_t>(vo);
-            if (lout_sys)
-              st_relaxed_sys(lout + r, e);
-            else
-              st_relaxed_gpu(lout + r, e);
-          }
-        }
-        vlast = Pv[K - 1];
       }
     }
     bulk_wait_all<0>();
