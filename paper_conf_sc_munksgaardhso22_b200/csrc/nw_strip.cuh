@@ -42,11 +42,18 @@
 
 namespace nwb200 {
 
-constexpr int kCH = 16;                    // rows per staging chunk (one bulk copy per lane)
-constexpr int kRefSlots = 5;               // ref ring: chunks Q-2 .. Q+2 live at event Q
-constexpr int kScSlots = 4;                // score ring: chunks Q-3 (being stored) .. Q
-constexpr int kRefRows = kRefSlots * kCH;  // 80
-constexpr int kScRows = kScSlots * kCH;    // 64
+// Ring geometry.  Events happen every kCH steps (event Q starts step kCH*Q).  In block Q lane t
+// touches rows kCH*Q+1-t .. kCH*Q+kCH-t, i.e. chunks Q-kSkewCh .. Q (the 31-row lane skew).
+constexpr int kCH = 16;                              // rows per staging chunk (<= 32, divides 32)
+constexpr int kSkewCh = (31 + kCH - 1) / kCH;        // chunks behind the newest one still in use
+constexpr int kLook = 2;                             // ref chunks fetched ahead (event Q issues Q+kLook)
+constexpr int kRefSlots = kLook + kSkewCh + 1;       // ref chunks live at once
+constexpr int kStoreDelay = kSkewCh + 1;             // chunk c complete after step kCH*c+kCH-1+31
+constexpr int kScSlots = kStoreDelay + 1;            // score chunks live (incl. the one being stored)
+constexpr int kRefRows = kRefSlots * kCH;
+constexpr int kScRows = kScSlots * kCH;
+constexpr int kSeqMod = 2 * kRefSlots;               // ref-chunk sequence modulus (slot + parity)
+static_assert(32 % kCH == 0, "events must align with the 32-row border windows");
 constexpr int kBarBytes = 128;
 constexpr unsigned kErrWatchdog = 0xBADB0001u;
 
@@ -112,7 +119,7 @@ __global__ void __launch_bounds__(32, 1) nw_strip_kernel(const StripParams P) {
   const int nch = (n + kCH - 1) / kCH;
   const int nsteps = n + 31;
   const int p = P.p;
-  int seq10 = 0;  // ref-chunk sequence number mod 10 (ring slot + mbarrier parity), kept across tasks
+  int seq10 = 0;  // ref-chunk sequence number mod kSeqMod (ring slot + mbarrier parity), across tasks
 
   for (;;) {
     unsigned long long tk = 0;
@@ -207,7 +214,7 @@ __global__ void __launch_bounds__(32, 1) nw_strip_kernel(const StripParams P) {
       int32_t* g = S + static_cast<long long>(r) * P.lds + c0;
       const uintptr_t gs = reinterpret_cast<uintptr_t>(g), ge = gs + 4u * ws;
       const uintptr_t as = (gs + 15) & ~static_cast<uintptr_t>(15), ae = ge & ~static_cast<uintptr_t>(15);
-      const int32_t* srow = sc_ring + ((r - 1) & (kScRows - 1)) * RS + static_cast<int>((gs >> 2) & 31);
+      const int32_t* srow = sc_ring + ((r - 1) % kScRows) * RS + static_cast<int>((gs >> 2) & 31);
       if (t < kCH) {
         if (ae > as) bulk_s2g(reinterpret_cast<void*>(as), smem_u32(srow) + static_cast<uint32_t>(as - gs),
                               static_cast<uint32_t>(ae - as));
@@ -236,7 +243,7 @@ __global__ void __launch_bounds__(32, 1) nw_strip_kernel(const StripParams P) {
     // per-lane incremental addressing for row r = step + 1 - t (starts at r0 = 1 - t)
     const int r0 = 1 - t;
     int ref_off = (((ref_row_base + r0 - 1) % kRefRows + kRefRows) % kRefRows) * RS;
-    int sc_off = ((r0 - 1) & (kScRows - 1)) * RS;
+    int sc_off = (((r0 - 1) % kScRows + kScRows) % kScRows) * RS;
     int gR = static_cast<int>((GR0 + static_cast<uintptr_t>(static_cast<intptr_t>(r0) * P.ldr)) & 31);
     int gS = static_cast<int>((GS0 + static_cast<uintptr_t>(static_cast<intptr_t>(r0) * P.lds)) & 31);
     uint64_t* lout_row = lout != nullptr ? lout + r0 : nullptr;
@@ -244,8 +251,7 @@ __global__ void __launch_bounds__(32, 1) nw_strip_kernel(const StripParams P) {
     const bool out_full = out_m == K - 1;
     fence_proxy_async();
     __syncwarp();
-    if (0 < nch) issue_ref(0);
-    if (1 < nch) issue_ref(1);
+    for (int c = 0; c < kLook && c < nch; ++c) issue_ref(c);
 
     // one wavefront step; ALL = every lane's row is in 1..n (steady state, no predicates)
     auto step = [&](const int sig, auto all_tag) {
@@ -319,21 +325,21 @@ __global__ void __launch_bounds__(32, 1) nw_strip_kernel(const StripParams P) {
       ++lout_row;
     };
 
-    for (int Q = 0; Q <= nch + 2; ++Q) {
+    for (int Q = 0; Q <= nch + kStoreDelay - 1; ++Q) {
       const int sig0 = Q * kCH;
       // ---- chunk events (warp-uniform)
-      if (Q >= 3 && Q - 3 < nch) {
-        fence_proxy_async();  // this lane's STS of rows in chunk Q-3 -> async proxy
+      bulk_wait_read<0>();  // stores issued at earlier events have read their slots
+      __syncwarp();
+      if (Q >= kStoreDelay && Q - kStoreDelay < nch) {
+        fence_proxy_async();  // this lane's STS of rows in the finished chunk -> async proxy
         __syncwarp();
-        store_sc(Q - 3);
+        store_sc(Q - kStoreDelay);
       }
       bulk_commit();
-      bulk_wait_read<1>();  // store of chunk Q-4 has read its slot; chunk Q may now reuse it
-      __syncwarp();
-      if (Q + 2 < nch) {
+      if (Q + kLook < nch) {
         fence_proxy_async();
         __syncwarp();
-        issue_ref(Q + 2);
+        issue_ref(Q + kLook);
       }
       if (Q < nch) mbar_wait(bar0 + 8 * ((seq10 + Q) % kRefSlots), ((seq10 + Q) / kRefSlots) & 1);
       if (sig0 >= nsteps) continue;
@@ -357,7 +363,7 @@ __global__ void __launch_bounds__(32, 1) nw_strip_kernel(const StripParams P) {
     }
     bulk_wait_all<0>();
     __syncwarp();
-    seq10 = (seq10 + nch) % 10;
+    seq10 = (seq10 + nch) % kSeqMod;
   }
 }
 
