@@ -186,7 +186,7 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu", action="store_true")
-    ap.add_argument("--variant", default="strip", choices=["strip", "diagonal", "unopt"],
+    ap.add_argument("--variant", default="strip", choices=["strip", "diagonal", "unopt", "seq"],
                     help="ablation: the paper's per-diagonal structure (Opt) / Unopt instead of the "
                          "persistent kernel")
     args = ap.parse_args()
@@ -228,7 +228,16 @@ def main():
         cells_local = nb * n * n
     else:
         S, R = inputs.device_problem(n, p, device=dev)
-        if args.variant == "strip":
+        if args.variant == "seq":       # NEXT-2: ref generated on chip from the sequences
+            a_h, b_h = inputs.gen_pair(n, inputs.SEED)
+            Ad, Bd = torch.from_numpy(a_h).to(dev), torch.from_numpy(b_h).to(dev)
+            tab = inputs.blosum62()
+            del R
+            R = None
+
+            def step():
+                nwb.nw_fill_seq(S, Ad, Bd, tab, p, tile)
+        elif args.variant == "strip":
             def step():
                 nwb.nw_fill(S, R, p, tile)
         else:
@@ -270,12 +279,14 @@ def main():
     value = cells_total / (ms_per_step * 1e-3) / 1e9
     # roofline of the (only) kernel: 8 algorithmic bytes per interior cell (ref read + score write)
     kern_ms = statistics.mean(per_launch)   # == the step: one launch per step for the strip kernel
-    achieved = 8.0 * cells_local / (kern_ms * 1e-3) / 1e9
+    bpc = 4.0 if args.variant == "seq" else 8.0   # algorithmic HBM bytes per cell
+    achieved = bpc * cells_local / (kern_ms * 1e-3) / 1e9
     peak, peak_src = measured_peaks()
     roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
             "traffic": ncu_traffic(cfg["workload"], tile), "peak_source": peak_src,
-            "algorithmic_bytes_per_launch": 8 * cells_local,
-            "kernel": ("nw_strip_kernel<%d>" % (4 if tile in (0, 128) else 2)) if args.variant == "strip"
+            "algorithmic_bytes_per_launch": int(bpc * cells_local),
+            "kernel": ("nw_strip_kernel<%d,%s>" % (4 if tile in (0, 128) else 2, args.variant == "seq"))
+            if args.variant in ("strip", "seq")
             else f"nw_diag_kernel<{tile}> x{nwb.nw_launch_count(1, n, tile)} launches (+copies: unopt)",
             "kernel_ms_mean": kern_ms, "kernel_ms_median": statistics.median(per_launch)}
     out = {"metric": METRIC, "value": value, "unit": "GCUPS", "n_gpus": world, "steps": args.steps,
@@ -287,11 +298,11 @@ def main():
                       "l2": "inputs %.1f GB >> 126 MB L2 (no flush needed)" % (8.0 * (n + 1) ** 2 * B / 1e9),
                       "parallelism": f"dp{world}" if world > 1 else "single"},
            "roofline": roof,
-           "gpu_launches": args.steps * nwb.nw_launch_count({"strip": 0, "diagonal": 1, "unopt": 2}[args.variant], n, tile),
+           "gpu_launches": args.steps * nwb.nw_launch_count({"strip": 0, "seq": 0, "diagonal": 1, "unopt": 2}[args.variant], n, tile),
            "variant": args.variant,
            "clocks": clk.summary()}
     # ---- e2e through the public C ABI with host buffers (H2D + kernel + D2H inside the timing)
-    if B == 1 and args.e2e_steps > 0:
+    if B == 1 and args.e2e_steps > 0 and args.variant == "strip":
         hs = torch.empty((n + 1, n + 1), dtype=torch.int32, pin_memory=True)
         hr = torch.empty((n + 1, n + 1), dtype=torch.int32, pin_memory=True)
         hr.copy_(R.cpu())

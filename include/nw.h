@@ -121,6 +121,22 @@ typedef struct {
 
 nw_status nw_fill_sharded(const nw_strip* strip, int32_t penalty, int32_t tile, void* stream);
 
+/* ---- NEXT-2: ref generated on chip from the two sequences --------------------------
+ * The step BEFORE the paper's path (Rodinia builds ref on the host): ref[i][j] =
+ * subst[a[i-1]][b[j-1]] is never materialised; each band keeps a packed int8 profile
+ * prof[x][lane] of its columns in shared memory.  HBM traffic drops from 8 to ~4 B/cell
+ * (the score write).  Result identical to nw_fill on the materialised ref.
+ * a, b     : DEVICE uint8 residue codes (< alphabet), n each (pair k at + k*stride_seq).
+ * subst    : HOST int32 alphabet x alphabet table (row-major, |v| <= 127), alphabet <= 32;
+ *            copied into the kernel parameters (no device allocation).
+ * Codes >= alphabet are memory-safe but give unspecified scores. */
+nw_status nw_fill_seq(int32_t* score, int64_t ld_score, const uint8_t* a, const uint8_t* b, int64_t n,
+                      const int32_t* subst, int32_t alphabet, int32_t penalty, int32_t tile, void* stream);
+nw_status nw_fill_seq_batch(int32_t* score, int64_t ld_score, int64_t stride_score, const uint8_t* a,
+                            const uint8_t* b, int64_t stride_seq, int64_t batch, int64_t n,
+                            const int32_t* subst, int32_t alphabet, int32_t penalty, int32_t tile,
+                            void* stream);
+
 /* ---- end to end from HOST memory (bench e2e) ---------------------------------------
  * Copies ref (rows 1..n) and the borders host->device, runs nw_fill, copies the full score
  * matrix device->host.  Host buffers: (n+1)x(n+1) int32, pitch n+1; pinned memory is

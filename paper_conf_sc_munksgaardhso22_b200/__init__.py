@@ -21,7 +21,7 @@ import threading
 from ._build import LIB_PATH, build  # noqa: F401  (build() is re-exported for __graft_entry__)
 
 __all__ = [
-    "NwError", "lib", "nw_fill", "nw_fill_batch", "nw_fill_sharded", "nw_fill_host",
+    "NwError", "lib", "nw_fill", "nw_fill_batch", "nw_fill_seq", "nw_fill_seq_batch", "nw_fill_sharded", "nw_fill_host",
     "nw_fill_diagonal", "nw_fill_unopt", "nw_band_width", "nw_launch_count", "nw_diag_lmad",
     "nw_kernel_info", "nw_strip_map", "nw_debug_set_grid", "nw_release_workspace", "nw_status_str",
 ]
@@ -73,6 +73,8 @@ def lib() -> ctypes.CDLL:
             L.nw_fill_batch.argtypes = [vp, vp, _i64, _i64, _i32, _i32, vp]
             L.nw_fill_batch_ld.argtypes = [vp, _i64, _i64, vp, _i64, _i64, _i64, _i64, _i32, _i32, vp]
             L.nw_fill_sharded.argtypes = [ctypes.POINTER(NwStrip), _i32, _i32, vp]
+            L.nw_fill_seq.argtypes = [vp, _i64, vp, vp, _i64, vp, _i32, _i32, _i32, vp]
+            L.nw_fill_seq_batch.argtypes = [vp, _i64, _i64, vp, vp, _i64, _i64, _i64, vp, _i32, _i32, _i32, vp]
             L.nw_fill_host.argtypes = [vp, vp, _i64, _i32, _i32, _i32]
             L.nw_fill_diagonal.argtypes = [vp, _i64, vp, _i64, _i64, _i32, _i32, vp]
             L.nw_fill_unopt.argtypes = [vp, _i64, vp, _i64, _i64, _i32, _i32, vp]
@@ -90,7 +92,8 @@ def lib() -> ctypes.CDLL:
             L.nw_debug_set_grid.restype = None
             L.nw_release_workspace.restype = None
             for f in ("nw_fill", "nw_fill_ld", "nw_fill_batch", "nw_fill_batch_ld", "nw_fill_sharded",
-                      "nw_fill_host", "nw_fill_diagonal", "nw_fill_unopt", "nw_kernel_info"):
+                      "nw_fill_host", "nw_fill_diagonal", "nw_fill_unopt", "nw_kernel_info", "nw_fill_seq",
+                      "nw_fill_seq_batch"):
                 getattr(L, f).restype = ctypes.c_int
             _lib = L
     return _lib
@@ -184,6 +187,48 @@ def nw_fill_sharded(score, ref, penalty: int, *, halo_in=None, halo_out=None, ep
     with torch.cuda.device(score.device):
         _check(lib().nw_fill_sharded(ctypes.byref(st), int(penalty), int(tile),
                                      _stream_ptr(stream, score.device)), "nw_fill_sharded")
+    return score
+
+
+def _subst_host(subst):
+    import numpy as np
+    t = np.ascontiguousarray(np.asarray(subst), dtype=np.int32)
+    if t.ndim != 2 or t.shape[0] != t.shape[1]:
+        raise ValueError("subst must be a square (alphabet x alphabet) table")
+    return t
+
+
+def nw_fill_seq(score, a, b, subst, penalty: int, tile: int = 0, stream=None):
+    """NEXT-2: fill score from the two sequences directly (ref never materialised).
+    score: int32 CUDA (n+1, >= n+1); a, b: uint8 CUDA (n,) residue codes; subst: host table."""
+    import torch
+    _mat(score, "score")
+    n = score.shape[0] - 1
+    for v, nm in ((a, "a"), (b, "b")):
+        if v.dtype != torch.uint8 or not v.is_cuda or v.dim() != 1 or v.numel() < n or v.stride(0) != 1:
+            raise ValueError(f"{nm} must be a contiguous uint8 CUDA vector of length >= n")
+    tab = _subst_host(subst)
+    with torch.cuda.device(score.device):
+        _check(lib().nw_fill_seq(score.data_ptr(), score.stride(0), a.data_ptr(), b.data_ptr(), n,
+                                 tab.ctypes.data, tab.shape[0], int(penalty), int(tile),
+                                 _stream_ptr(stream, score.device)), "nw_fill_seq")
+    return score
+
+
+def nw_fill_seq_batch(score, a, b, subst, penalty: int, tile: int = 0, stream=None):
+    """Batch NEXT-2: score (B, n+1, >= n+1) int32; a, b (B, n) uint8 CUDA, contiguous rows."""
+    import torch
+    _mat(score, "score")
+    B, n = score.shape[0], score.shape[1] - 1
+    if a.shape != b.shape or a.dim() != 2 or a.shape[0] != B or a.shape[1] < n or a.dtype != torch.uint8 \
+            or b.dtype != torch.uint8 or a.stride(1) != 1 or b.stride(1) != 1 or a.stride(0) != b.stride(0):
+        raise ValueError("a, b must be (B, >= n) uint8 CUDA tensors with equal strides")
+    tab = _subst_host(subst)
+    with torch.cuda.device(score.device):
+        _check(lib().nw_fill_seq_batch(score.data_ptr(), score.stride(1), score.stride(0), a.data_ptr(),
+                                       b.data_ptr(), a.stride(0), B, n, tab.ctypes.data, tab.shape[0],
+                                       int(penalty), int(tile), _stream_ptr(stream, score.device)),
+               "nw_fill_seq_batch")
     return score
 
 

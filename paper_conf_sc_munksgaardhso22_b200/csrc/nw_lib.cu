@@ -66,8 +66,16 @@ nw_status check_range(int64_t n, int32_t p) {
 struct DevInfo {
   bool init = false;
   int sms = 0;
-  int occ2 = 0, occ4 = 0;
+  int occ[2][2] = {{0, 0}, {0, 0}};  // [K==4][SEQ]
 };
+
+template <int K, bool SEQ>
+cudaError_t setup_kernel(int* occ) {
+  cudaError_t e = cudaFuncSetAttribute(nw_strip_kernel<K, SEQ>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       static_cast<int>(StripGeom<K, SEQ>::kSmem));
+  if (e != cudaSuccess) return e;
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, nw_strip_kernel<K, SEQ>, 32, StripGeom<K, SEQ>::kSmem);
+}
 
 std::mutex g_mu;
 DevInfo g_dev[128];
@@ -78,13 +86,13 @@ nw_status dev_info(int dev, DevInfo** out) {
   DevInfo& d = g_dev[dev];
   if (!d.init) {
     NW_CU(cudaDeviceGetAttribute(&d.sms, cudaDevAttrMultiProcessorCount, dev));
-    NW_CU(cudaFuncSetAttribute(nw_strip_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                               static_cast<int>(StripGeom<2>::kSmem)));
-    NW_CU(cudaFuncSetAttribute(nw_strip_kernel<4>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                               static_cast<int>(StripGeom<4>::kSmem)));
-    NW_CU(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ2, nw_strip_kernel<2>, 32, StripGeom<2>::kSmem));
-    NW_CU(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&d.occ4, nw_strip_kernel<4>, 32, StripGeom<4>::kSmem));
-    if (d.occ2 < 1 || d.occ4 < 1) return cuda_fail(cudaErrorInvalidConfiguration);
+    NW_CU((setup_kernel<2, false>(&d.occ[0][0])));
+    NW_CU((setup_kernel<2, true>(&d.occ[0][1])));
+    NW_CU((setup_kernel<4, false>(&d.occ[1][0])));
+    NW_CU((setup_kernel<4, true>(&d.occ[1][1])));
+    for (auto& r : d.occ)
+      for (int o : r)
+        if (o < 1) return cuda_fail(cudaErrorInvalidConfiguration);
     d.init = true;
   }
   *out = &d;
@@ -148,8 +156,11 @@ unsigned long long spin_limit_ns() {
 // One launch of the persistent kernel over `pairs` x ceil(width/W) bands.
 nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* ref, int64_t ldr, int64_t psr,
                        int64_t pairs, int64_t n, int64_t width, int32_t p, int32_t tile, const uint64_t* halo_in,
-                       uint64_t* halo_out, uint32_t halo_epoch, int32_t halo_out_sys, cudaStream_t st) {
+                       uint64_t* halo_out, uint32_t halo_epoch, int32_t halo_out_sys, cudaStream_t st,
+                       const uint8_t* seq_a = nullptr, const uint8_t* seq_b = nullptr, int64_t psa = 0,
+                       int64_t psb = 0, const int8_t* subst32 = nullptr) {
   const int K = tile_to_k(tile);
+  const bool SEQ = seq_a != nullptr;
   const int W = 32 * K;
   if (pairs == 0 || n == 0 || width == 0) return NW_OK;
   int dev = 0;
@@ -186,16 +197,28 @@ nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* 
   P.ticket = w->d_ticket;
   P.err = w->d_err;
   P.spin_limit_ns = spin_limit_ns();
-  const int occ = K == 2 ? di->occ2 : di->occ4;
+  if (SEQ) {
+    P.seq_a = seq_a;
+    P.seq_b = seq_b;
+    P.psa = psa;
+    P.psb = psb;
+    for (int i = 0; i < 32 * 32; ++i) P.subst[i] = subst32[i];
+  }
+  const int occ = di->occ[K == 4][SEQ];
   int64_t grid = static_cast<int64_t>(occ) * di->sms;
   if (g_debug_grid > 0) grid = g_debug_grid;
   if (grid > P.ntasks) grid = P.ntasks;
   P.ticket_base = w->ticket_next;
   w->ticket_next += static_cast<unsigned long long>(P.ntasks + grid);  // every CTA draws one extra ticket
-  if (K == 2)
-    nw_strip_kernel<2><<<static_cast<unsigned>(grid), 32, StripGeom<2>::kSmem, st>>>(P);
+  const unsigned g = static_cast<unsigned>(grid);
+  if (K == 2 && !SEQ)
+    nw_strip_kernel<2, false><<<g, 32, StripGeom<2, false>::kSmem, st>>>(P);
+  else if (K == 2)
+    nw_strip_kernel<2, true><<<g, 32, StripGeom<2, true>::kSmem, st>>>(P);
+  else if (!SEQ)
+    nw_strip_kernel<4, false><<<g, 32, StripGeom<4, false>::kSmem, st>>>(P);
   else
-    nw_strip_kernel<4><<<static_cast<unsigned>(grid), 32, StripGeom<4>::kSmem, st>>>(P);
+    nw_strip_kernel<4, true><<<g, 32, StripGeom<4, true>::kSmem, st>>>(P);
   NW_CU(cudaGetLastError());
   return NW_OK;
 }
@@ -336,6 +359,31 @@ nw_status nw_fill_sharded(const nw_strip* sp, int32_t penalty, int32_t tile, voi
                       S.halo_out, S.epoch, S.halo_out_is_peer, static_cast<cudaStream_t>(stream));
 }
 
+nw_status nw_fill_seq_batch(int32_t* score, int64_t ld_score, int64_t stride_score, const uint8_t* a,
+                            const uint8_t* b, int64_t stride_seq, int64_t batch, int64_t n, const int32_t* subst,
+                            int32_t alphabet, int32_t penalty, int32_t tile, void* stream) {
+  if (batch < 0 || !score || !a || !b || !subst || n < 0 || n > kMaxN || tile_to_k(tile) == 0) return NW_EINVAL;
+  if (alphabet < 1 || alphabet > 32 || ld_score < n + 1 || !aligned4(score)) return NW_EINVAL;
+  const int64_t ss = span_bytes(n, ld_score) / 4;
+  if (batch > 1 && (stride_score < ss || stride_seq < n)) return NW_EINVAL;
+  int8_t tab[32 * 32] = {0};
+  for (int x = 0; x < alphabet; ++x)
+    for (int y = 0; y < alphabet; ++y) {
+      const int32_t v = subst[x * alphabet + y];
+      if (v < -128 || v > 127) return NW_ERANGE;
+      tab[x * 32 + y] = static_cast<int8_t>(v);
+    }
+  nw_status s = check_range(n, penalty);
+  if (s != NW_OK || batch == 0 || n == 0) return s;
+  return launch_strip(score, ld_score, stride_score, nullptr, 0, 0, batch, n, n, penalty, tile, nullptr, nullptr, 0,
+                      0, static_cast<cudaStream_t>(stream), a, b, stride_seq, stride_seq, tab);
+}
+
+nw_status nw_fill_seq(int32_t* score, int64_t ld_score, const uint8_t* a, const uint8_t* b, int64_t n,
+                      const int32_t* subst, int32_t alphabet, int32_t penalty, int32_t tile, void* stream) {
+  return nw_fill_seq_batch(score, ld_score, 0, a, b, 0, 1, n, subst, alphabet, penalty, tile, stream);
+}
+
 nw_status nw_fill_host(int32_t* score_host, const int32_t* ref_host, int64_t n, int32_t penalty, int32_t tile,
                        int32_t device) {
   if (!score_host || !ref_host || n < 0 || n > kMaxN || tile_to_k(tile) == 0) return NW_EINVAL;
@@ -414,14 +462,14 @@ nw_status nw_kernel_info(int32_t tile, int32_t device, int64_t* smem_bytes, int3
                          int32_t* num_sms) {
   const int K = tile_to_k(tile);
   if (!K) return NW_EINVAL;
-  if (smem_bytes) *smem_bytes = static_cast<int64_t>(K == 2 ? StripGeom<2>::kSmem : StripGeom<4>::kSmem);
+  if (smem_bytes) *smem_bytes = static_cast<int64_t>(K == 2 ? StripGeom<2, false>::kSmem : StripGeom<4, false>::kSmem);
   if (!ctas_per_sm && !num_sms) return NW_OK;
   NW_CU(cudaSetDevice(device));
   std::lock_guard<std::mutex> lk(g_mu);
   DevInfo* di = nullptr;
   nw_status s = dev_info(device, &di);
   if (s != NW_OK) return s;
-  if (ctas_per_sm) *ctas_per_sm = K == 2 ? di->occ2 : di->occ4;
+  if (ctas_per_sm) *ctas_per_sm = di->occ[K == 4][0];
   if (num_sms) *num_sms = di->sms;
   return NW_OK;
 }

@@ -57,11 +57,13 @@ static_assert(32 % kCH == 0, "events must align with the 32-row border windows")
 constexpr int kBarBytes = 128;
 constexpr unsigned kErrWatchdog = 0xBADB0001u;
 
-template <int K>
+template <int K, bool SEQ = false>
 struct StripGeom {
   static constexpr int W = 32 * K;   // band width (columns)
   static constexpr int RS = W + 36;  // row slot (words): W + 3 head + 3 tail + 28 swizzle, 16B multiple
-  static constexpr size_t kSmem = kBarBytes + 4ull * (size_t)(kRefRows + kScRows) * RS;
+  static constexpr int kProfWords = 32 * 32;  // SEQ: prof[x][lane] = K packed int8 subst[x][b_j]
+  static constexpr size_t kSmem =
+      kBarBytes + 4ull * ((SEQ ? 0 : (size_t)kRefRows * RS) + (size_t)kScRows * RS + (SEQ ? kProfWords : 0));
   static_assert(RS % 4 == 0, "row slots must be 16-byte multiples for cp.async.bulk");
   static_assert((kRefRows * RS) % 32 == 0 && (kScRows * RS) % 32 == 0, "ring wrap must keep banks");
 };
@@ -96,18 +98,30 @@ struct StripParams {
   unsigned long long ticket_base;
   unsigned int* err;
   unsigned long long spin_limit_ns;
+  // NEXT-2 (SEQ kernels): ref[i][j] = subst[a[i-1]][b[j-1]] generated on chip
+  const uint8_t* seq_a;
+  const uint8_t* seq_b;
+  int64_t psa, psb;  // pair strides of a / b (bytes)
+  int8_t subst[32 * 32];
 };
 
-template <int K>
-__global__ void __launch_bounds__(32, 1) nw_strip_kernel(const StripParams P) {
-  using G = StripGeom<K>;
+__device__ __forceinline__ int prmt_sext(uint32_t w, uint32_t sel) {
+  uint32_t d;
+  asm("prmt.b32 %0, %1, 0, %2;" : "=r"(d) : "r"(w), "r"(sel));
+  return static_cast<int>(d);
+}
+
+template <int K, bool SEQ>
+__global__ void __launch_bounds__(32, 1) nw_strip_kernel(const __grid_constant__ StripParams P) {
+  using G = StripGeom<K, SEQ>;
   constexpr int RS = G::RS;
   constexpr unsigned FULL = 0xffffffffu;
   extern __shared__ __align__(128) unsigned char smem[];
   const int t = threadIdx.x;
   const uint32_t bar0 = smem_u32(smem);
   int32_t* const ref_ring = reinterpret_cast<int32_t*>(smem + kBarBytes);
-  int32_t* const sc_ring = ref_ring + kRefRows * RS;
+  int32_t* const sc_ring = ref_ring + (SEQ ? 0 : kRefRows * RS);
+  uint32_t* const prof = reinterpret_cast<uint32_t*>(sc_ring + kScRows * RS);
 
   if (t == 0) {
     for (int i = 0; i < kRefSlots; ++i) mbar_init(bar0 + 8 * i, 32);
@@ -251,7 +265,27 @@ __global__ void __launch_bounds__(32, 1) nw_strip_kernel(const StripParams P) {
     const bool out_full = out_m == K - 1;
     fence_proxy_async();
     __syncwarp();
-    for (int c = 0; c < kLook && c < nch; ++c) issue_ref(c);
+    if constexpr (!SEQ) {
+      for (int c = 0; c < kLook && c < nch; ++c) issue_ref(c);
+    }
+    // SEQ: per-band substitution profile prof[x][t] = pack_m subst[x][b[c0-1+tK+m]] (int8 x K)
+    const uint8_t* const A = SEQ ? P.seq_a + pair * P.psa : nullptr;
+    int a0 = 0, a1 = 0;  // residues of this lane's current and next row (software pipeline)
+    if constexpr (SEQ) {
+      const uint8_t* const Bq = P.seq_b + pair * P.psb;
+      int bj[K];
+#pragma unroll
+      for (int m = 0; m < K; ++m) bj[m] = (t * K + m < ws) ? (Bq[c0 - 1 + t * K + m] & 31) : 0;
+      for (int x = 0; x < 32; ++x) {
+        uint32_t w = 0;
+#pragma unroll
+        for (int m = 0; m < K; ++m) w |= static_cast<uint32_t>(static_cast<uint8_t>(P.subst[x * 32 + bj[m]])) << (8 * m);
+        prof[x * 32 + t] = w;
+      }
+      a0 = A[min(max(r0 - 1, 0), n - 1)] & 31;
+      a1 = A[min(max(r0, 0), n - 1)] & 31;
+      __syncwarp();
+    }
 
     // one wavefront step; ALL = every lane's row is in 1..n (steady state, no predicates)
     auto step = [&](const int sig, auto all_tag) {
@@ -284,11 +318,17 @@ __global__ void __launch_bounds__(32, 1) nw_strip_kernel(const StripParams P) {
         active = r >= 1 && r <= n;
       }
       if (active) {
-        const int32_t* rrow = ref_ring + ref_off + gR + t * K;
         int32_t* srow = sc_ring + sc_off + gS + t * K;
         int rv[K];
+        if constexpr (SEQ) {
+          const uint32_t pw = prof[a0 * 32 + t];
 #pragma unroll
-        for (int m = 0; m < K; ++m) rv[m] = rrow[m];
+          for (int m = 0; m < K; ++m) rv[m] = prmt_sext(pw, 0x8880u + 0x1111u * m);  // sign-extended byte m
+        } else {
+          const int32_t* rrow = ref_ring + ref_off + gR + t * K;
+#pragma unroll
+          for (int m = 0; m < K; ++m) rv[m] = rrow[m];
+        }
         int d = Lprev, l = L;
 #pragma unroll
         for (int m = 0; m < K; ++m) {
@@ -316,6 +356,10 @@ __global__ void __launch_bounds__(32, 1) nw_strip_kernel(const StripParams P) {
       }
       vlast = Pv[K - 1];
       // advance this lane to row r+1
+      if constexpr (SEQ) {
+        a0 = a1;
+        a1 = __ldg(A + min(max(lane_row(sig, t) + 1, 0), n - 1)) & 31;  // residue of row r+2
+      }
       ref_off += RS;
       if (ref_off >= kRefRows * RS) ref_off -= kRefRows * RS;
       sc_off += RS;
@@ -336,12 +380,12 @@ __global__ void __launch_bounds__(32, 1) nw_strip_kernel(const StripParams P) {
         store_sc(Q - kStoreDelay);
       }
       bulk_commit();
-      if (Q + kLook < nch) {
+      if (!SEQ && Q + kLook < nch) {
         fence_proxy_async();
         __syncwarp();
         issue_ref(Q + kLook);
       }
-      if (Q < nch) mbar_wait(bar0 + 8 * ((seq10 + Q) % kRefSlots), ((seq10 + Q) / kRefSlots) & 1);
+      if (!SEQ && Q < nch) mbar_wait(bar0 + 8 * ((seq10 + Q) % kRefSlots), ((seq10 + Q) / kRefSlots) & 1);
       if (sig0 >= nsteps) continue;
       if ((sig0 & 31) == 0 && sig0 > 0) {
         cur = nxt;

@@ -200,3 +200,38 @@ def test_full_size_configs_bit_exact(n, tile):
     nwb.nw_fill(s_dev, r_dev, p, tile)
     torch.cuda.synchronize()
     _stream_compare(s_dev, score[0], ref, n, p)
+
+
+@pytest.mark.parametrize("tile", [0, 64])
+@pytest.mark.parametrize("n", [1, 5, 31, 64, 129, 1000, 4096])
+def test_fill_seq_next2(n, tile):
+    """NEXT-2: ref generated on chip from (a, b, BLOSUM62) == nw_fill on the materialised ref."""
+    a, b = inputs.gen_pair(n, 100 + n)
+    ref = inputs.build_ref(a, b)
+    score = inputs.init_borders(inputs.aligned_matrix(n), 10)
+    inputs.fill_interior(score, inputs.SENTINEL)
+    want = expect(score, ref, 10)
+    s = to_dev(score)
+    nwb.nw_fill_seq(s, torch.from_numpy(a).cuda(), torch.from_numpy(b).cuda(), inputs.blosum62(), 10, tile)
+    torch.cuda.synchronize()
+    np.testing.assert_array_equal(s.cpu().numpy(), want)
+
+
+def test_fill_seq_batch_next2():
+    B, n = 6, 300
+    pairs = [inputs.gen_pair(n, inputs.pair_seed(k)) for k in range(B)]
+    want = []
+    S = np.empty((B, n + 1, n + 1), dtype=np.int32)
+    for k, (a, b) in enumerate(pairs):
+        s0 = inputs.init_borders(inputs.aligned_matrix(n), 10)
+        inputs.fill_interior(s0, inputs.SENTINEL)
+        S[k] = s0
+        want.append(expect(s0, inputs.build_ref(a, b), 10))
+    Sd = torch.from_numpy(S).cuda()
+    Ad = torch.from_numpy(np.stack([a for a, _ in pairs])).cuda()
+    Bd = torch.from_numpy(np.stack([b for _, b in pairs])).cuda()
+    nwb.nw_fill_seq_batch(Sd, Ad, Bd, inputs.blosum62(), 10, 0)
+    torch.cuda.synchronize()
+    got = Sd.cpu().numpy()
+    for k in range(B):
+        np.testing.assert_array_equal(got[k], want[k], err_msg=f"pair {k}")
