@@ -235,3 +235,25 @@ def test_fill_seq_batch_next2():
     got = Sd.cpu().numpy()
     for k in range(B):
         np.testing.assert_array_equal(got[k], want[k], err_msg=f"pair {k}")
+
+
+def test_config4_shape_batch_bit_exact():
+    """BASELINE.json config 4 shape (n=2048 pairs seeded 7 ^ k*C) on 512 pairs, built on the device
+    as bench.py builds them, every cell checked with the oracle (threads: ctypes drops the GIL)."""
+    from concurrent.futures import ThreadPoolExecutor
+    n, p, B = 2048, 10, 512
+    S = torch.empty((B, n + 1, n + 1), dtype=torch.int32, device="cuda")
+    R = torch.empty((B, n + 1, n + 1), dtype=torch.int32, device="cuda")
+    for k in range(B):
+        inputs.device_problem(n, p, seed=inputs.pair_seed(k), device="cuda", score=S[k], ref=R[k])
+    nwb.nw_fill_batch(S, R, p, 0)
+    torch.cuda.synchronize()
+    got = S.cpu().numpy()
+
+    def check(k):
+        s, r = inputs.make_problem(n, p, seed=inputs.pair_seed(k))
+        return bool(np.array_equal(got[k], oracle.nw_ref(s, r, p)))
+
+    with ThreadPoolExecutor(8) as ex:
+        ok = list(ex.map(check, range(B)))
+    assert all(ok), [k for k, v in enumerate(ok) if not v][:10]
