@@ -100,7 +100,8 @@ nw_status nw_fill_batch_ld(int32_t* score, int64_t ld_score, int64_t stride_scor
  *            (entry i = (epoch << 32) | (uint32) score[i][col0]); NULL on rank 0.
  *            Must be zero-filled once before first use; never needs resetting after.
  * halo_out : rank g+1's halo_in (a peer-mapped pointer, e.g. torch symmetric memory) or
- *            NULL on the last rank.  Written with st.relaxed.sys, one entry per row as soon
+ *            NULL on the last rank.  A rank with halo_out needs w % nw_band_width(tile) == 0
+ *            (else NW_ECOMM).  Written with st.relaxed.sys, one entry per row as soon
  *            as the row's last column is final — the NVLink border push is fused into the
  *            wavefront kernel (no host involvement, no separate send/recv).
  * epoch    : nonzero, identical on all ranks for one collective call, strictly increasing

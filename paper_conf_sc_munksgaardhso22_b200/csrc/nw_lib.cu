@@ -353,6 +353,8 @@ nw_status nw_fill_sharded(const nw_strip* sp, int32_t penalty, int32_t tile, voi
   if ((S.halo_in && (reinterpret_cast<uintptr_t>(S.halo_in) & 7)) ||
       (S.halo_out && (reinterpret_cast<uintptr_t>(S.halo_out) & 7)))
     return NW_ECOMM;
+  // a strip that pushes a halo must end on a band boundary (its last band is then full width)
+  if (S.halo_out && S.w % nw_band_width(tile) != 0) return NW_ECOMM;
   nw_status s = check_range(S.n > S.w ? S.n : S.w, penalty);
   if (s != NW_OK || S.n == 0 || S.w == 0) return s;
   return launch_strip(S.score, S.ld_score, 0, S.ref, S.ld_ref, 0, 1, S.n, S.w, penalty, tile, S.halo_in,

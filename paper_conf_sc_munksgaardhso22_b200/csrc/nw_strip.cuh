@@ -174,7 +174,7 @@ __global__ void __launch_bounds__(32, 1) nw_strip_kernel(const __grid_constant__
       lout_epoch = P.halo_epoch;
     }
     const int32_t* const colp = S + (c0 - 1);  // plain left border column (band 0 without halo)
-    const int out_lane = (ws - 1) / K, out_m = (ws - 1) % K;
+    const int out_lane = (ws - 1) / K;
     const int ref_row_base = (seq10 % kRefSlots) * kCH;
     // Row slots are swizzled by the row's own global word address: element x of row r sits at
     // slot(r) + (G(r) & 31) + x, G(r) = word address of (r, c0).  The 16-byte phase G & 3 keeps
@@ -262,7 +262,6 @@ __global__ void __launch_bounds__(32, 1) nw_strip_kernel(const __grid_constant__
     int gS = static_cast<int>((GS0 + static_cast<uintptr_t>(static_cast<intptr_t>(r0) * P.lds)) & 31);
     uint64_t* lout_row = lout != nullptr ? lout + r0 : nullptr;
     const bool do_out = lout != nullptr && t == out_lane;
-    const bool out_full = out_m == K - 1;
     fence_proxy_async();
     __syncwarp();
     if constexpr (!SEQ) {
@@ -342,12 +341,9 @@ __global__ void __launch_bounds__(32, 1) nw_strip_kernel(const __grid_constant__
 #pragma unroll
         for (int m = 0; m < K; ++m) srow[m] = Pv[m];
         if (do_out) {
-          int vo = Pv[K - 1];
-          if (!out_full) {
-#pragma unroll
-            for (int m = 0; m < K - 1; ++m)
-              if (m == out_m) vo = Pv[m];
-          }
+          // the publishing lane holds the band's last column in Pv[K-1]: every band with a right
+          // neighbour is full width (only a pair's / the last rank's final band is ragged)
+          const int vo = Pv[K - 1];
           if (lout_sys)
             st_relaxed_sys_v2(lout_row, static_cast<uint32_t>(vo), lout_epoch);
           else

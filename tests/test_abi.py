@@ -124,3 +124,17 @@ def test_band_width_and_launch_counts():
     assert nwb.nw_launch_count(1, 32768, 16) == 2 * 2048 - 1         # Rodinia: one per diagonal
     assert nwb.nw_launch_count(2, 32768, 16) == 2 * (2 * 2048 - 1)   # Unopt: + one copy each
     assert nwb.nw_launch_count(1, 1000, 16) == 2 * 63 - 1            # ragged q = ceil(n/b)
+
+
+def test_sharded_halo_strip_must_end_on_band(L):
+    # w = 100 is not a multiple of the band width: pushing a halo from it is rejected
+    s = NwStrip(FAKE_S, 101, FAKE_R, 101, 64, 100, None, 0x20000000, 3, 1)
+    assert L.nw_fill_sharded(ctypes.byref(s), 10, 0, None) == NW_ECOMM
+    if not _has_gpu():   # last rank (no halo_out): valid; without a GPU it must fail in CUDA, not compute
+        s = NwStrip(FAKE_S, 101, FAKE_R, 101, 64, 100, 0x20000000, None, 3, 0)
+        assert L.nw_fill_sharded(ctypes.byref(s), 10, 0, None) == NW_ECUDA
+
+
+def _has_gpu():
+    import torch
+    return torch.cuda.is_available()
