@@ -31,6 +31,7 @@ CONFIGS = {
     2: dict(workload="nw_n16384_p10", n=16384, batch=1, tile=64),
     3: dict(workload="nw_n32768_p10", n=32768, batch=1, tile=0),
     4: dict(workload="nw_batch4096_n2048_p10", n=2048, batch=4096, tile=0),
+    5: dict(workload="nw_n65536_p10_strips", n=65536, batch=1, tile=0, strips=True),
 }
 PENALTY = 10
 METRIC = "NW GCUPS (interior cell updates / s), bit-exact vs CPU oracle"
@@ -213,10 +214,21 @@ def main():
         dist.init_process_group("nccl", device_id=dev)
     n, p, tile = cfg["n"], PENALTY, cfg["tile"]
     B = cfg["batch"]
-    if B > 1:
-        per = B // world
-        lo = rank * per
-        hi = B if rank == world - 1 else lo + per
+    strips = cfg.get("strips", False) and world > 1
+    if strips:
+        # config 5: column strips of one n=65536 pair, right border pushed to the next rank over
+        # NVLink from inside the kernel (torch symmetric memory peer pointers), one barrier per call
+        from paper_conf_sc_munksgaardhso22_b200 import dist as nwdist
+        shard = nwdist.StripShard(n, p, inputs.SEED, tile=tile)
+        S = shard.score
+
+        def step():
+            shard.fill()
+            shard.barrier()
+        cells_local = n * shard.strip.w
+    elif B > 1:
+        from paper_conf_sc_munksgaardhso22_b200 import dist as nwdist
+        lo, hi = nwdist.pair_range(B, world, rank)
         nb = hi - lo
         S = torch.empty((nb, n + 1, n + 1), dtype=torch.int32, device=dev)
         R = torch.empty((nb, n + 1, n + 1), dtype=torch.int32, device=dev)
@@ -274,7 +286,7 @@ def main():
         tt = torch.tensor([total_ms], device=dev)
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         total_ms = float(tt.item())
-    cells_total = cells_local if world == 1 else B * n * n
+    cells_total = cells_local if world == 1 else B * n * n   # (strips: B = 1, all n*n cells)
     ms_per_step = total_ms / args.steps
     value = cells_total / (ms_per_step * 1e-3) / 1e9
     # roofline of the (only) kernel: 8 algorithmic bytes per interior cell (ref read + score write)
@@ -296,13 +308,13 @@ def main():
            "config": {"workload": cfg["workload"], "n": n, "batch": B, "penalty": p, "tile": tile,
                       "band_width": nwb.nw_band_width(tile), "pairs_per_rank": B // world if B > 1 else 1,
                       "l2": "inputs %.1f GB >> 126 MB L2 (no flush needed)" % (8.0 * (n + 1) ** 2 * B / 1e9),
-                      "parallelism": f"dp{world}" if world > 1 else "single"},
+                      "parallelism": (f"strips{world}" if strips else f"dp{world}") if world > 1 else "single"},
            "roofline": roof,
            "gpu_launches": args.steps * nwb.nw_launch_count({"strip": 0, "seq": 0, "diagonal": 1, "unopt": 2}[args.variant], n, tile),
            "variant": args.variant,
            "clocks": clk.summary()}
     # ---- e2e through the public C ABI with host buffers (H2D + kernel + D2H inside the timing)
-    if B == 1 and args.e2e_steps > 0 and args.variant == "strip":
+    if B == 1 and args.e2e_steps > 0 and args.variant == "strip" and not strips:
         hs = torch.empty((n + 1, n + 1), dtype=torch.int32, pin_memory=True)
         hr = torch.empty((n + 1, n + 1), dtype=torch.int32, pin_memory=True)
         hr.copy_(R.cpu())
@@ -323,7 +335,7 @@ def main():
         del hs, hr
     elif B > 1:
         out["e2e"] = None
-    gpu_last = S[n].cpu().numpy() if B == 1 else None
+    gpu_last = S[n].cpu().numpy() if B == 1 and not strips else None
     if rank == 0 and not args.no_cpu:
         out["cpu_baseline"] = cpu_baseline(cfg, gpu_last)
     if rank == 0:
