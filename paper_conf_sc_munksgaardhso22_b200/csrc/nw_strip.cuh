@@ -256,10 +256,15 @@ __global__ void __launch_bounds__(32, 1) nw_strip_kernel(const __grid_constant__
     bool wvalid = window_valid();
     // per-lane incremental addressing for row r = step + 1 - t (starts at r0 = 1 - t)
     const int r0 = 1 - t;
-    int ref_off = (((ref_row_base + r0 - 1) % kRefRows + kRefRows) % kRefRows) * RS;
-    int sc_off = (((r0 - 1) % kScRows + kScRows) % kScRows) * RS;
+    // 32-bit shared byte addresses of this lane's first column in its current row:
+    //   ring + 4*(row_slot*RS + (G(r) & 31) + t*K); one add + two wrap fix-ups per step.
     int gR = static_cast<int>((GR0 + static_cast<uintptr_t>(static_cast<intptr_t>(r0) * P.ldr)) & 31);
     int gS = static_cast<int>((GS0 + static_cast<uintptr_t>(static_cast<intptr_t>(r0) * P.lds)) & 31);
+    const uint32_t refR0 = smem_u32(ref_ring), refR1 = refR0 + 4u * kRefRows * RS;
+    const uint32_t scR0 = smem_u32(sc_ring), scR1 = scR0 + 4u * kScRows * RS;
+    uint32_t aR = refR0 + 4u * ((((ref_row_base + r0 - 1) % kRefRows + kRefRows) % kRefRows) * RS + gR + t * K);
+    uint32_t aS = scR0 + 4u * ((((r0 - 1) % kScRows + kScRows) % kScRows) * RS + gS + t * K);
+    const uint32_t stepR = 4u * (RS + ldr32), stepS = 4u * (RS + lds32);
     uint64_t* lout_row = lout != nullptr ? lout + r0 : nullptr;
     const bool do_out = lout != nullptr && t == out_lane;
     fence_proxy_async();
@@ -317,16 +322,15 @@ __global__ void __launch_bounds__(32, 1) nw_strip_kernel(const __grid_constant__
         active = r >= 1 && r <= n;
       }
       if (active) {
-        int32_t* srow = sc_ring + sc_off + gS + t * K;
+
         int rv[K];
         if constexpr (SEQ) {
           const uint32_t pw = prof[a0 * 32 + t];
 #pragma unroll
           for (int m = 0; m < K; ++m) rv[m] = prmt_sext(pw, 0x8880u + 0x1111u * m);  // sign-extended byte m
         } else {
-          const int32_t* rrow = ref_ring + ref_off + gR + t * K;
 #pragma unroll
-          for (int m = 0; m < K; ++m) rv[m] = rrow[m];
+          for (int m = 0; m < K; ++m) rv[m] = lds_s32(aR + 4 * m);
         }
         int d = Lprev, l = L;
 #pragma unroll
@@ -339,7 +343,7 @@ __global__ void __launch_bounds__(32, 1) nw_strip_kernel(const __grid_constant__
         }
         Lprev = L;
 #pragma unroll
-        for (int m = 0; m < K; ++m) srow[m] = Pv[m];
+        for (int m = 0; m < K; ++m) sts_s32(aS + 4 * m, Pv[m]);
         if (do_out) {
           // the publishing lane holds the band's last column in Pv[K-1]: every band with a right
           // neighbour is full width (only a pair's / the last rank's final band is ragged)
@@ -356,12 +360,20 @@ __global__ void __launch_bounds__(32, 1) nw_strip_kernel(const __grid_constant__
         a0 = a1;
         a1 = __ldg(A + min(max(lane_row(sig, t) + 1, 0), n - 1)) & 31;  // residue of row r+2
       }
-      ref_off += RS;
-      if (ref_off >= kRefRows * RS) ref_off -= kRefRows * RS;
-      sc_off += RS;
-      if (sc_off >= kScRows * RS) sc_off -= kScRows * RS;
-      gR = (gR + ldr32) & 31;
-      gS = (gS + lds32) & 31;
+      aR += stepR;  // next row slot + swizzle advance (G(r+1) = G(r) + ld)
+      gR += ldr32;
+      if (gR >= 32) {
+        gR -= 32;
+        aR -= 128;
+      }
+      if (aR >= refR1) aR -= refR1 - refR0;
+      aS += stepS;
+      gS += lds32;
+      if (gS >= 32) {
+        gS -= 32;
+        aS -= 128;
+      }
+      if (aS >= scR1) aS -= scR1 - scR0;
       ++lout_row;
     };
 
