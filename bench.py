@@ -187,6 +187,7 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--trace", default="", help="write per-band {task,start,end,smid} of one extra launch here (.npy)")
     ap.add_argument("--variant", default="strip", choices=["strip", "diagonal", "unopt", "seq"],
                     help="ablation: the paper's per-diagonal structure (Opt) / Unopt instead of the "
                          "persistent kernel")
@@ -313,6 +314,14 @@ def main():
            "gpu_launches": args.steps * nwb.nw_launch_count({"strip": 0, "seq": 0, "diagonal": 1, "unopt": 2}[args.variant], n, tile),
            "variant": args.variant,
            "clocks": clk.summary()}
+    if args.trace and not strips:
+        ntask = (B if B > 1 else 1) * -(-n // nwb.nw_band_width(tile))
+        tb = torch.zeros((ntask, 4), dtype=torch.int64, device=dev)
+        nwb.nw_debug_set_trace(tb)
+        step()
+        torch.cuda.synchronize()
+        nwb.nw_debug_set_trace(None)
+        np.save(args.trace, tb.cpu().numpy())
     # ---- e2e through the public C ABI with host buffers (H2D + kernel + D2H inside the timing)
     if B == 1 and args.e2e_steps > 0 and args.variant == "strip" and not strips:
         hs = torch.empty((n + 1, n + 1), dtype=torch.int32, pin_memory=True)

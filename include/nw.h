@@ -185,6 +185,11 @@ nw_status nw_kernel_info(int32_t tile, int32_t device, int64_t* smem_bytes, int3
  * occupancy).  A 1-CTA grid must still finish (ticket order => deadlock freedom). */
 void nw_debug_set_grid(int32_t grid);
 
+/* Debug hook: persistent-kernel launches record, per task (pair, band) t < cap_tasks, four
+ * uint64 {t, start_ns, end_ns, smid} (%globaltimer) into the DEVICE buffer dev_buf (NULL = off).
+ * Used by bench.py --trace to measure the wavefront ramp and the band-to-band lag. */
+void nw_debug_set_trace(uint64_t* dev_buf, int64_t cap_tasks);
+
 /* Frees every cached workspace (device buffers, pinned staging).  Not thread-safe with
  * concurrent nw_* calls. */
 void nw_release_workspace(void);

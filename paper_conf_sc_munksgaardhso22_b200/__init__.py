@@ -23,7 +23,7 @@ from ._build import LIB_PATH, build  # noqa: F401  (build() is re-exported for _
 __all__ = [
     "NwError", "lib", "nw_fill", "nw_fill_batch", "nw_fill_seq", "nw_fill_seq_batch", "nw_fill_sharded", "nw_fill_host",
     "nw_fill_diagonal", "nw_fill_unopt", "nw_band_width", "nw_launch_count", "nw_diag_lmad",
-    "nw_kernel_info", "nw_strip_map", "nw_debug_set_grid", "nw_release_workspace", "nw_status_str",
+    "nw_kernel_info", "nw_strip_map", "nw_debug_set_grid", "nw_debug_set_trace", "nw_release_workspace", "nw_status_str",
 ]
 
 NW_OK, NW_EINVAL, NW_ERANGE, NW_ECUDA, NW_ENOMEM, NW_ECOMM = range(6)
@@ -88,6 +88,8 @@ def lib() -> ctypes.CDLL:
                                          ctypes.POINTER(_i32)]
             L.nw_strip_map.argtypes = [_i64, _i64, _i32, _i32, _i32, _i32, ctypes.POINTER(_i64)]
             L.nw_strip_map.restype = _i32
+            L.nw_debug_set_trace.argtypes = [vp, _i64]
+            L.nw_debug_set_trace.restype = None
             L.nw_debug_set_grid.argtypes = [_i32]
             L.nw_debug_set_grid.restype = None
             L.nw_release_workspace.restype = None
@@ -298,6 +300,14 @@ def nw_kernel_info(tile: int = 0, device: int = 0):
 
 def nw_debug_set_grid(grid: int):
     lib().nw_debug_set_grid(int(grid))
+
+
+def nw_debug_set_trace(buf=None):
+    """buf: int64 CUDA tensor of shape (>= tasks, 4) or None (off)."""
+    if buf is None:
+        lib().nw_debug_set_trace(None, 0)
+    else:
+        lib().nw_debug_set_trace(buf.data_ptr(), buf.shape[0])
 
 
 def nw_release_workspace():

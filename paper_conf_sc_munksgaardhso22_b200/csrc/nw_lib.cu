@@ -80,6 +80,8 @@ cudaError_t setup_kernel(int* occ) {
 std::mutex g_mu;
 DevInfo g_dev[128];
 int g_debug_grid = 0;
+unsigned long long* g_trace = nullptr;
+long long g_trace_cap = 0;
 
 nw_status dev_info(int dev, DevInfo** out) {
   if (dev < 0 || dev >= 128) return NW_EINVAL;
@@ -197,6 +199,8 @@ nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* 
   P.ticket = w->d_ticket;
   P.err = w->d_err;
   P.spin_limit_ns = spin_limit_ns();
+  P.trace = g_trace;
+  P.trace_cap = g_trace_cap;
   if (SEQ) {
     P.seq_a = seq_a;
     P.seq_b = seq_b;
@@ -494,6 +498,12 @@ int32_t nw_strip_map(int64_t n, int64_t width, int32_t tile, int32_t band, int32
 }
 
 void nw_debug_set_grid(int32_t grid) { g_debug_grid = grid > 0 ? grid : 0; }
+
+void nw_debug_set_trace(uint64_t* dev_buf, int64_t cap_tasks) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  g_trace = reinterpret_cast<unsigned long long*>(dev_buf);
+  g_trace_cap = dev_buf ? cap_tasks : 0;
+}
 
 void nw_release_workspace(void) {
   std::lock_guard<std::mutex> lk(g_mu);

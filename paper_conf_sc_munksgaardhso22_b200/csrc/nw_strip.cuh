@@ -98,6 +98,8 @@ struct StripParams {
   unsigned long long ticket_base;
   unsigned int* err;
   unsigned long long spin_limit_ns;
+  unsigned long long* trace;  // debug: per task {task, t_start, t_end, smid} (globaltimer ns) or null
+  long long trace_cap;
   // NEXT-2 (SEQ kernels): ref[i][j] = subst[a[i-1]][b[j-1]] generated on chip
   const uint8_t* seq_a;
   const uint8_t* seq_b;
@@ -141,6 +143,7 @@ __global__ void __launch_bounds__(32, 1) nw_strip_kernel(const __grid_constant__
     tk = __shfl_sync(FULL, tk, 0);
     const long long task = static_cast<long long>(tk - P.ticket_base);
     if (task >= P.ntasks) break;
+    const unsigned long long t_task0 = globaltimer_ns();
     const long long pair = task / P.nbands;
     const int band = static_cast<int>(task - pair * P.nbands);
     const bool last_band = band == P.nbands - 1;
@@ -416,6 +419,15 @@ __global__ void __launch_bounds__(32, 1) nw_strip_kernel(const __grid_constant__
     bulk_wait_all<0>();
     __syncwarp();
     seq10 = (seq10 + nch) % kSeqMod;
+    if (P.trace != nullptr && t == 0 && task < P.trace_cap) {
+      unsigned smid;
+      asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+      unsigned long long* e = P.trace + 4 * task;
+      e[0] = static_cast<unsigned long long>(task);
+      e[1] = t_task0;
+      e[2] = globaltimer_ns();
+      e[3] = smid;
+    }
   }
 }
 
