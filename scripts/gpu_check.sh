@@ -1,5 +1,6 @@
 #!/bin/bash
 # One gpurun call: smoke, GPU parity tests, bench (headline + ablations), ncu launch list + full capture.
+export NW_SPIN_LIMIT_MS=10000
 set -x
 mkdir -p gpurun_out
 nvidia-smi --query-gpu=name,clocks.max.sm,memory.total --format=csv
