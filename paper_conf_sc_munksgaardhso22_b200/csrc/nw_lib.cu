@@ -37,7 +37,7 @@ constexpr int64_t kMaxN = (int64_t{1} << 30) - 64;
 
 int tile_to_k(int32_t tile) {
   switch (tile) {
-    case 0: return 4;
+    case 0: return 2;
     case 16:
     case 32:
     case 64: return 2;
@@ -63,18 +63,25 @@ nw_status check_range(int64_t n, int32_t p) {
   return NW_OK;
 }
 
+// Kernel instances: K columns per lane, NW warps (bands) per CTA, CH-row staging chunks,
+// LOOK chunks of ref prefetch (DESIGN.md §4.3 sizes the rings).
+using CfgK2 = StripCfg<2, false, 4, 8, 3>;
+using CfgK2S = StripCfg<2, true, 4, 8, 3>;
+using CfgK4 = StripCfg<4, false, 2, 16, 2>;
+using CfgK4S = StripCfg<4, true, 2, 16, 2>;
+
 struct DevInfo {
   bool init = false;
   int sms = 0;
   int occ[2][2] = {{0, 0}, {0, 0}};  // [K==4][SEQ]
 };
 
-template <int K, bool SEQ>
+template <class C>
 cudaError_t setup_kernel(int* occ) {
-  cudaError_t e = cudaFuncSetAttribute(nw_strip_kernel<K, SEQ>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       static_cast<int>(StripGeom<K, SEQ>::kSmem));
+  cudaError_t e = cudaFuncSetAttribute(nw_strip_kernel<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       static_cast<int>(C::kSmem));
   if (e != cudaSuccess) return e;
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, nw_strip_kernel<K, SEQ>, 32, StripGeom<K, SEQ>::kSmem);
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, nw_strip_kernel<C>, 32 * C::NW, C::kSmem);
 }
 
 std::mutex g_mu;
@@ -88,10 +95,10 @@ nw_status dev_info(int dev, DevInfo** out) {
   DevInfo& d = g_dev[dev];
   if (!d.init) {
     NW_CU(cudaDeviceGetAttribute(&d.sms, cudaDevAttrMultiProcessorCount, dev));
-    NW_CU((setup_kernel<2, false>(&d.occ[0][0])));
-    NW_CU((setup_kernel<2, true>(&d.occ[0][1])));
-    NW_CU((setup_kernel<4, false>(&d.occ[1][0])));
-    NW_CU((setup_kernel<4, true>(&d.occ[1][1])));
+    NW_CU((setup_kernel<CfgK2>(&d.occ[0][0])));
+    NW_CU((setup_kernel<CfgK2S>(&d.occ[0][1])));
+    NW_CU((setup_kernel<CfgK4>(&d.occ[1][0])));
+    NW_CU((setup_kernel<CfgK4S>(&d.occ[1][1])));
     for (auto& r : d.occ)
       for (int o : r)
         if (o < 1) return cuda_fail(cudaErrorInvalidConfiguration);
@@ -190,6 +197,8 @@ nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* 
   P.p = p;
   P.nbands = static_cast<int32_t>(nbands);
   P.ntasks = pairs * nbands;
+  const int NW = K == 2 ? CfgK2::NW : CfgK4::NW;
+  P.ngroups = (P.ntasks + NW - 1) / NW;
   P.xbuf = w->xbuf;
   P.epoch = ++w->epoch;
   P.halo_in = halo_in;
@@ -211,18 +220,18 @@ nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* 
   const int occ = di->occ[K == 4][SEQ];
   int64_t grid = static_cast<int64_t>(occ) * di->sms;
   if (g_debug_grid > 0) grid = g_debug_grid;
-  if (grid > P.ntasks) grid = P.ntasks;
+  if (grid > P.ngroups) grid = P.ngroups;
   P.ticket_base = w->ticket_next;
-  w->ticket_next += static_cast<unsigned long long>(P.ntasks + grid);  // every CTA draws one extra ticket
+  w->ticket_next += static_cast<unsigned long long>(P.ngroups + grid);  // every CTA draws one extra ticket
   const unsigned g = static_cast<unsigned>(grid);
   if (K == 2 && !SEQ)
-    nw_strip_kernel<2, false><<<g, 32, StripGeom<2, false>::kSmem, st>>>(P);
+    nw_strip_kernel<CfgK2><<<g, 32 * CfgK2::NW, CfgK2::kSmem, st>>>(P);
   else if (K == 2)
-    nw_strip_kernel<2, true><<<g, 32, StripGeom<2, true>::kSmem, st>>>(P);
+    nw_strip_kernel<CfgK2S><<<g, 32 * CfgK2S::NW, CfgK2S::kSmem, st>>>(P);
   else if (!SEQ)
-    nw_strip_kernel<4, false><<<g, 32, StripGeom<4, false>::kSmem, st>>>(P);
+    nw_strip_kernel<CfgK4><<<g, 32 * CfgK4::NW, CfgK4::kSmem, st>>>(P);
   else
-    nw_strip_kernel<4, true><<<g, 32, StripGeom<4, true>::kSmem, st>>>(P);
+    nw_strip_kernel<CfgK4S><<<g, 32 * CfgK4S::NW, CfgK4S::kSmem, st>>>(P);
   NW_CU(cudaGetLastError());
   return NW_OK;
 }
@@ -468,7 +477,7 @@ nw_status nw_kernel_info(int32_t tile, int32_t device, int64_t* smem_bytes, int3
                          int32_t* num_sms) {
   const int K = tile_to_k(tile);
   if (!K) return NW_EINVAL;
-  if (smem_bytes) *smem_bytes = static_cast<int64_t>(K == 2 ? StripGeom<2, false>::kSmem : StripGeom<4, false>::kSmem);
+  if (smem_bytes) *smem_bytes = static_cast<int64_t>(K == 2 ? CfgK2::kSmem : CfgK4::kSmem);
   if (!ctas_per_sm && !num_sms) return NW_OK;
   NW_CU(cudaSetDevice(device));
   std::lock_guard<std::mutex> lk(g_mu);
