@@ -316,7 +316,7 @@ def main():
            "clocks": clk.summary()}
     if args.trace and not strips:
         ntask = (B if B > 1 else 1) * -(-n // nwb.nw_band_width(tile))
-        tb = torch.zeros((ntask, 4), dtype=torch.int64, device=dev)
+        tb = torch.zeros((ntask, 8), dtype=torch.int64, device=dev)
         nwb.nw_debug_set_trace(tb)
         step()
         torch.cuda.synchronize()

@@ -185,8 +185,9 @@ nw_status nw_kernel_info(int32_t tile, int32_t device, int64_t* smem_bytes, int3
  * occupancy).  A 1-CTA grid must still finish (ticket order => deadlock freedom). */
 void nw_debug_set_grid(int32_t grid);
 
-/* Debug hook: persistent-kernel launches record, per task (pair, band) t < cap_tasks, four
- * uint64 {t, start_ns, end_ns, smid} (%globaltimer) into the DEVICE buffer dev_buf (NULL = off).
+/* Debug hook: persistent-kernel launches record, per task (pair, band) t < cap_tasks, eight
+ * uint64 {t, start_ns, end_ns, smid, event_cycles, ref_wait_cycles, border_spin_cycles,
+ * total_cycles} into the DEVICE buffer dev_buf (NULL = off).
  * Used by bench.py --trace to measure the wavefront ramp and the band-to-band lag. */
 void nw_debug_set_trace(uint64_t* dev_buf, int64_t cap_tasks);
 

@@ -303,7 +303,7 @@ def nw_debug_set_grid(grid: int):
 
 
 def nw_debug_set_trace(buf=None):
-    """buf: int64 CUDA tensor of shape (>= tasks, 4) or None (off)."""
+    """buf: int64 CUDA tensor of shape (>= tasks, 8) or None (off)."""
     if buf is None:
         lib().nw_debug_set_trace(None, 0)
     else:

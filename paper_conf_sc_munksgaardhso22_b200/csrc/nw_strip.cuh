@@ -222,6 +222,7 @@ __global__ void __launch_bounds__(32 * C::NW, 1) nw_strip_kernel(const __grid_co
     const uint32_t gen = static_cast<uint32_t>(gcount & 3) << 30;
     if (task < P.ntasks) {
       const unsigned long long t_task0 = globaltimer_ns();
+      const long long c_task0 = clock64();
       const long long pair = task / P.nbands;
       const int band = static_cast<int>(task - pair * P.nbands);
       const bool last_band = band == P.nbands - 1;
@@ -388,6 +389,8 @@ __global__ void __launch_bounds__(32 * C::NW, 1) nw_strip_kernel(const __grid_co
       }
       const uint32_t* const profp = prof + t;
       uint32_t tok = 0;  // produced by each chunk's mbarrier wait, consumed by the ref loads
+      const bool tracing = P.trace != nullptr;
+      long long ev_cyc = 0, spin_cyc = 0, wait_cyc = 0;  // debug cycle accounting (trace only)
 
       // one wavefront step; ALL = every lane's row is in 1..n (steady state, no predicates)
       auto step = [&](const int sig, auto all_tag, auto src_tag) {
@@ -409,11 +412,13 @@ __global__ void __launch_bounds__(32 * C::NW, 1) nw_strip_kernel(const __grid_co
           uint64_t be = lds64_volatile(bring_in + 8u * ((sig + 1) & (kBR - 1)));
           const uint32_t want = gen | static_cast<uint32_t>(sig + 1);
           if (static_cast<uint32_t>(be >> 32) != want && sig < n) {
+            const long long c_0 = clock64();
             const uint64_t t0 = globaltimer_ns();
             do {
               be = lds64_volatile(bring_in + 8u * ((sig + 1) & (kBR - 1)));
               if (globaltimer_ns() - t0 > P.spin_limit_ns) watchdog_trap(P.err);
             } while (static_cast<uint32_t>(be >> 32) != want);
+            spin_cyc += clock64() - c_0;
           }
           bval = static_cast<int>(static_cast<uint32_t>(be));
         } else {
@@ -422,6 +427,7 @@ __global__ void __launch_bounds__(32 * C::NW, 1) nw_strip_kernel(const __grid_co
           if (!wvalid) {
             uint32_t bep = __shfl_sync(FULL, static_cast<uint32_t>(cur >> 32), idx);
             if (bep != lin_epoch && sig < n) {  // left band has not published row sig+1 yet
+              const long long c_0 = clock64();
               const int rowb = win_base + t;
               const uint64_t t0 = globaltimer_ns();
               for (;;) {
@@ -432,6 +438,7 @@ __global__ void __launch_bounds__(32 * C::NW, 1) nw_strip_kernel(const __grid_co
               }
               bval = __shfl_sync(FULL, static_cast<int>(static_cast<uint32_t>(cur)), idx);
               wvalid = window_valid();
+              spin_cyc += clock64() - c_0;
             }
           }
         }
@@ -506,6 +513,7 @@ __global__ void __launch_bounds__(32 * C::NW, 1) nw_strip_kernel(const __grid_co
 
       for (int Q = 0; Q <= nch + C::STORE_DELAY - 1; ++Q) {
         const int sig0 = Q * CH;
+        const long long c_ev0 = tracing ? clock64() : 0;
         // ---- chunk events (warp-uniform)
         bulk_wait_read<0>();  // stores issued at earlier events have read their slots
         __syncwarp();
@@ -521,7 +529,9 @@ __global__ void __launch_bounds__(32 * C::NW, 1) nw_strip_kernel(const __grid_co
             __syncwarp();
             issue_ref(Q + C::LOOK);
           }
+          const long long c_w0 = tracing ? clock64() : 0;
           if (Q < nch) tok = mbar_wait_tok(bar0 + 8 * ((seqm + Q) % C::REF_SLOTS), ((seqm + Q) / C::REF_SLOTS) & 1);
+          if (tracing) wait_cyc += clock64() - c_w0;
         }
         if (sig0 >= nsteps) continue;
         if (src == kSrcSmem) {
@@ -544,6 +554,7 @@ __global__ void __launch_bounds__(32 * C::NW, 1) nw_strip_kernel(const __grid_co
             }
           }
         }
+        if (tracing) ev_cyc += clock64() - c_ev0;
         if (src == kSrcSmem)
           run_block(sig0, std::true_type{});
         else
@@ -555,11 +566,15 @@ __global__ void __launch_bounds__(32 * C::NW, 1) nw_strip_kernel(const __grid_co
       if (P.trace != nullptr && t == 0 && task < P.trace_cap) {
         unsigned smid;
         asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
-        unsigned long long* e = P.trace + 4 * task;
+        unsigned long long* e = P.trace + 8 * task;
         e[0] = static_cast<unsigned long long>(task);
         e[1] = t_task0;
         e[2] = globaltimer_ns();
         e[3] = smid;
+        e[4] = static_cast<unsigned long long>(ev_cyc);    // cycles in chunk events (incl. ref wait)
+        e[5] = static_cast<unsigned long long>(wait_cyc);  // of which: ref mbarrier waits
+        e[6] = static_cast<unsigned long long>(spin_cyc);  // cycles spinning on the left border
+        e[7] = static_cast<unsigned long long>(clock64() - c_task0);
       }
     }
     __syncthreads();  // group end: every warp done (shared border rings / progress reusable)

@@ -29,6 +29,15 @@ def main(path, n=None):
     act = [int(((st <= g) & (en > g)).sum()) for g in grid]
     print("bands in flight over the launch:", act)
     print("distinct SMs:", len(np.unique(t[:, 3])))
+    if t.shape[1] >= 8:
+        tot = t[:, 7].astype(float)
+        for name, col in (("events", 4), ("ref waits", 5), ("border spins", 6)):
+            fr = t[:, col] / np.maximum(tot, 1)
+            print(f"  {name:13s}: mean {fr.mean()*100:5.1f}% of task cycles (band0 {fr[0]*100:5.1f}%)")
+        if n:
+            comp = (tot - t[:, 4] - t[:, 6]) / n
+            print(f"  step cycles/row excluding events+spins: mean {comp.mean():.1f}, band0 {comp[0]:.1f};"
+                  f" total cycles/row band0 {tot[0]/n:.1f}")
 
 
 if __name__ == "__main__":
