@@ -1,8 +1,8 @@
 // nw_ptx.cuh — thin inline-PTX wrappers for sm_100a used by the NW kernels.
 //
-// Bulk async copies (cp.async.bulk, SASS UBLKCP) move whole row segments between global
-// memory and shared memory; mbarrier transaction counts track the loads; bulk groups track
-// the stores.  Relaxed 64-bit loads/stores carry the epoch-tagged border entries (single-copy
+// Row segments move between global and shared memory with 16-byte cp.async (LDGSTS, completion
+// on an mbarrier) and LDS.128/STG.128 (the per-row cp.async.bulk variants are kept for
+// reference; small bulk copies serialise in the TMA unit).  Relaxed 64-bit loads/stores carry the epoch-tagged border entries (single-copy
 // atomic for aligned 8-byte accesses, PTX memory model), at GPU scope within a device and at
 // system scope across NVLink peers.
 #pragma once
@@ -21,6 +21,27 @@ __device__ __forceinline__ int lds_s32(uint32_t a) {
 }
 __device__ __forceinline__ void sts_s32(uint32_t a, int v) {
   asm volatile("st.shared.b32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+
+// 16-byte asynchronous global->shared copy through L2 only (LDGSTS), and a 4-byte one
+__device__ __forceinline__ void cp_async16(uint32_t dst, const void* src) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async4(uint32_t dst, const void* src) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(dst), "l"(src) : "memory");
+}
+// arrive on `bar` once this thread's prior cp.async copies have landed (counts toward the
+// arrival count given at init)
+__device__ __forceinline__ void cp_async_arrive(uint32_t bar) {
+  asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(bar) : "memory");
+}
+__device__ __forceinline__ int4 lds128(uint32_t a) {
+  int4 v;
+  asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ void stg128(void* p, int4 v) {
+  asm volatile("st.global.v4.b32 [%0], {%1, %2, %3, %4};" ::"l"(p), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w) : "memory");
 }
 
 __device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {

@@ -51,7 +51,7 @@ def test_library_is_sm100a_only():
     assert "sm_100a" in out
     sass = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "-sass", nwb.LIB_PATH],
                           capture_output=True, text=True).stdout
-    assert "UBLKCP" in sass          # cp.async.bulk staging (TMA bulk engine)
+    assert "LDGSTS" in sass          # cp.async staging of the ref rows (LSU async copies)
     assert "VIADDMNMX" in sass       # DPX add+max cell update
 
 
