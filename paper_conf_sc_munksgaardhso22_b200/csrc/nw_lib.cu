@@ -210,6 +210,7 @@ nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* 
   P.spin_limit_ns = spin_limit_ns();
   P.trace = g_trace;
   P.trace_cap = g_trace_cap;
+  P.trace2 = g_trace ? g_trace + 8 * g_trace_cap : nullptr;
   if (SEQ) {
     P.seq_a = seq_a;
     P.seq_b = seq_b;

@@ -111,6 +111,7 @@ struct StripParams {
   unsigned long long spin_limit_ns;
   unsigned long long* trace;  // debug: per task 8 x u64 (see nw.h nw_debug_set_trace) or null
   long long trace_cap;
+  unsigned long long* trace2;  // debug: per task {store cycles, ref-issue cycles} or null
   // NEXT-2 (SEQ kernels): ref[i][j] = subst[a[i-1]][b[j-1]] generated on chip
   const uint8_t* seq_a;
   const uint8_t* seq_b;
@@ -196,6 +197,7 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
   const long long c_task0 = clock64();
   const bool tracing = P.trace != nullptr;
   long long ev_cyc = 0, spin_cyc = 0, wait_cyc = 0;  // debug cycle accounting (trace only)
+  long long st_cyc = 0, is_cyc = 0;
 
   const uint32_t s_prog = smem_u32(smem + 8);
   const uint32_t s_bring = smem_u32(smem + 128);
@@ -452,8 +454,11 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
     const long long c_ev0 = tracing ? clock64() : 0;
     // ---- chunk events (warp-uniform)
     if (Q >= C::STORE_DELAY && Q - C::STORE_DELAY < nch) store_sc(Q - C::STORE_DELAY);
+    const long long c_st1 = tracing ? clock64() : 0;
+    if (tracing) st_cyc += c_st1 - c_ev0;
     if constexpr (!SEQ) {
       if (Q + C::LOOK < nch) issue_ref(Q + C::LOOK);
+      if (tracing) is_cyc += clock64() - c_st1;
       if (Q < nch) {
         const long long c_w0 = tracing ? clock64() : 0;
         const int sl = Q % C::SLOTS;
@@ -528,6 +533,11 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
     e[5] = static_cast<unsigned long long>(wait_cyc);  // of which: ref mbarrier waits
     e[6] = static_cast<unsigned long long>(spin_cyc);  // of which: left-border spins
     e[7] = static_cast<unsigned long long>(clock64() - c_task0);
+    if (P.trace_cap < 0) return;
+  }
+  if (P.trace != nullptr && t == 0 && task < P.trace_cap && P.trace2 != nullptr) {
+    P.trace2[2 * task] = static_cast<unsigned long long>(st_cyc);
+    P.trace2[2 * task + 1] = static_cast<unsigned long long>(is_cyc);
   }
 }
 

@@ -11,7 +11,7 @@ import numpy as np
 
 def main(path, n=None):
     t = np.load(path).astype(np.int64)
-    t = t[t[:, 2] > 0]
+    t = t[t[:, 2] > 0].astype(np.int64)
     t = t[np.argsort(t[:, 0])]
     t0 = t[:, 1].min()
     st, en = (t[:, 1] - t0) / 1e3, (t[:, 2] - t0) / 1e3   # us
@@ -31,11 +31,14 @@ def main(path, n=None):
     print("distinct SMs:", len(np.unique(t[:, 3])))
     if t.shape[1] >= 8:
         tot = t[:, 7].astype(float)
-        for name, col in (("events", 4), ("ref waits", 5), ("border spins", 6)):
+        cols = [("events", 4), ("ref waits", 5), ("border spins", 6)]
+        if t.shape[1] >= 10:
+            cols += [("score stores", 8), ("ref issue", 9)]
+        for name, col in cols:
             fr = t[:, col] / np.maximum(tot, 1)
             print(f"  {name:13s}: mean {fr.mean()*100:5.1f}% of task cycles (band0 {fr[0]*100:5.1f}%)")
         if n:
-            comp = (tot - t[:, 4] - t[:, 6]) / n
+            comp = (tot - t[:, 4]) / n
             print(f"  step cycles/row excluding events+spins: mean {comp.mean():.1f}, band0 {comp[0]:.1f};"
                   f" total cycles/row band0 {tot[0]/n:.1f}")
 
