@@ -35,6 +35,34 @@ __device__ __forceinline__ void cp_async4(uint32_t dst, const void* src) {
 __device__ __forceinline__ void cp_async_arrive(uint32_t bar) {
   asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(bar) : "memory");
 }
+// predicated forms (no branch): p == false -> no access
+__device__ __forceinline__ void cp_async16_p(bool p, uint32_t dst, const void* src) {
+  asm volatile("{ .reg .pred q; setp.ne.b32 q, %0, 0; @q cp.async.cg.shared.global [%1], [%2], 16; }" ::"r"(static_cast<int>(p)),
+               "r"(dst), "l"(src)
+               : "memory");
+}
+__device__ __forceinline__ int4 lds128_p(bool p, uint32_t a) {
+  int4 v = make_int4(0, 0, 0, 0);
+  asm volatile("{ .reg .pred q; setp.ne.b32 q, %4, 0; @q ld.shared.v4.b32 {%0, %1, %2, %3}, [%5]; }"
+               : "+r"(v.x), "+r"(v.y), "+r"(v.z), "+r"(v.w)
+               : "r"(static_cast<int>(p)), "r"(a)
+               : "memory");
+  return v;
+}
+__device__ __forceinline__ void stg128_p(bool p, void* ptr, int4 v) {
+  asm volatile("{ .reg .pred q; setp.ne.b32 q, %0, 0; @q st.global.v4.b32 [%1], {%2, %3, %4, %5}; }" ::"r"(static_cast<int>(p)),
+               "l"(ptr), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w)
+               : "memory");
+}
+__device__ __forceinline__ int lds32_p(bool p, uint32_t a) {
+  int v = 0;
+  asm volatile("{ .reg .pred q; setp.ne.b32 q, %1, 0; @q ld.shared.b32 %0, [%2]; }" : "+r"(v) : "r"(static_cast<int>(p)), "r"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ void stg32_p(bool p, void* ptr, int v) {
+  asm volatile("{ .reg .pred q; setp.ne.b32 q, %0, 0; @q st.global.b32 [%1], %2; }" ::"r"(static_cast<int>(p)), "l"(ptr), "r"(v)
+               : "memory");
+}
 __device__ __forceinline__ int4 lds128(uint32_t a) {
   int4 v;
   asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a) : "memory");

@@ -277,69 +277,80 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
     return true;
   };
 
-  // ref chunk c (rows CH*c+1 .. CH*c+CH): 16-byte cp.async over (row, chunk) pairs, then every
+  // Per-lane staging assignments, fixed for the whole task: in iteration it lane t moves the
+  // 16-byte chunk k of row i of a CH-row chunk (f = t + 32*it, i = f / MAX, k = f % MAX).
+  // Row addresses advance by CH*ld per chunk; with CH a multiple of 4 and ld odd the 16-byte
+  // phase of row i is the same in every chunk.
+  const char* const Rb = reinterpret_cast<const char*>(R);
+  char* const Sb = reinterpret_cast<char*>(S);
+  // ref chunk c (rows CH*c+1 .. CH*c+CH): straight-line predicated cp.async (LDGSTS), then every
   // lane arrives on the chunk's mbarrier when its copies have landed.
   auto issue_ref = [&](int c) {
-#pragma unroll 1
+    const long long row0 = static_cast<long long>(c) * CH + 1;
+#pragma unroll
     for (int it = 0; it < C::ITER_R; ++it) {
       const int f = t + 32 * it;
       const int i = f / C::MAXR, k = f - (f / C::MAXR) * C::MAXR;
-      const int r = c * CH + 1 + i;
-      if (i < CH && r <= n) {
-        const uintptr_t gs = reinterpret_cast<uintptr_t>(R + static_cast<long long>(r) * P.ldr + c0);
-        const uintptr_t s0 = gs & ~static_cast<uintptr_t>(15);
-        const uintptr_t e0 = (gs + 4u * ws + 15) & ~static_cast<uintptr_t>(15);
-        const uintptr_t ca = s0 + 16u * k;
-        if (ca < e0) {
-          const uint32_t dst =
-              refR0 + 4u * (((r - 1) & (kRing - 1)) * RS + static_cast<int>((gs >> 2) & 28)) + 16u * k;
-          if (ca + 16 <= rend) {
-            cp_async16(dst, reinterpret_cast<const void*>(ca));
-          } else {  // the matrix's last row: never read past its final element
-            for (int x = 0; x < 4; ++x)
-              if (ca + 4u * x < rend) cp_async4(dst + 4u * x, reinterpret_cast<const void*>(ca + 4u * x));
-          }
-        }
+      const int r = static_cast<int>(row0) + i;
+      const uintptr_t gs = reinterpret_cast<uintptr_t>(Rb) + 4u * static_cast<uintptr_t>((row0 + i) * P.ldr + c0);
+      const uintptr_t ca = (gs & ~static_cast<uintptr_t>(15)) + 16u * k;
+      const uintptr_t e0 = (gs + 4u * ws + 15) & ~static_cast<uintptr_t>(15);
+      const uint32_t dst = refR0 + 4u * (((r - 1) & (kRing - 1)) * RS + static_cast<int>((gs >> 2) & 28)) + 16u * k;
+      const bool in = i < CH && r <= n && ca < e0;
+      cp_async16_p(in && ca + 16 <= rend, dst, reinterpret_cast<const void*>(ca));
+      if (in && ca + 16 > rend) {  // the matrix's last row: never read past its final element
+        for (int x = 0; x < 4; ++x)
+          if (ca + 4u * x < rend) cp_async4(dst + 4u * x, reinterpret_cast<const void*>(ca + 4u * x));
       }
     }
     cp_async_arrive(bar0 + 8 * (c % C::SLOTS));
   };
 
-  // score chunk c: LDS.128 + STG.128 of the aligned interiors, scalar head/tail words
+  // score chunk c: all LDS.128 first, then all STG.128 (aligned interiors); scalar head/tail
+  // words (<= 3 each) by lanes 0..2CH-1
   auto store_sc = [&](int c) {
-#pragma unroll 1
+    const long long row0 = static_cast<long long>(c) * CH + 1;
+    int4 v[C::ITER_S];
+    uintptr_t dst[C::ITER_S];
+    bool ok[C::ITER_S];
+#pragma unroll
     for (int it = 0; it < C::ITER_S; ++it) {
       const int f = t + 32 * it;
       const int i = f / C::MAXS, k = f - (f / C::MAXS) * C::MAXS;
-      const int r = c * CH + 1 + i;
-      if (i < CH && r <= n) {
-        const uintptr_t gs = reinterpret_cast<uintptr_t>(S + static_cast<long long>(r) * P.lds + c0);
-        const uintptr_t ge = gs + 4u * ws;
-        const uintptr_t as = (gs + 15) & ~static_cast<uintptr_t>(15), ae = ge & ~static_cast<uintptr_t>(15);
-        const uintptr_t ca = as + 16u * k;
-        if (ca < ae) {
-          const uint32_t srow = scR0 + 4u * (((r - 1) & (kRing - 1)) * RS + static_cast<int>((gs >> 2) & 31));
-          stg128(reinterpret_cast<void*>(ca), lds128(srow + static_cast<uint32_t>(ca - gs)));
-        }
-      }
+      const int r = static_cast<int>(row0) + i;
+      const uintptr_t gs = reinterpret_cast<uintptr_t>(Sb) + 4u * static_cast<uintptr_t>((row0 + i) * P.lds + c0);
+      const uintptr_t as = (gs + 15) & ~static_cast<uintptr_t>(15), ae = (gs + 4u * ws) & ~static_cast<uintptr_t>(15);
+      dst[it] = as + 16u * k;
+      ok[it] = i < CH && r <= n && dst[it] < ae;
+      const uint32_t srow = scR0 + 4u * (((r - 1) & (kRing - 1)) * RS + static_cast<int>((gs >> 2) & 31));
+      v[it] = lds128_p(ok[it], srow + static_cast<uint32_t>(dst[it] - gs));
     }
+#pragma unroll
+    for (int it = 0; it < C::ITER_S; ++it) stg128_p(ok[it], reinterpret_cast<void*>(dst[it]), v[it]);
     {  // lanes 0..CH-1: head words of row t; lanes CH..2CH-1: tail words of row t-CH
       const int i = t % CH;
-      const int r = c * CH + 1 + i;
-      if (t < 2 * CH && r <= n) {
-        int32_t* g = S + static_cast<long long>(r) * P.lds + c0;
-        const uintptr_t gs = reinterpret_cast<uintptr_t>(g), ge = gs + 4u * ws;
-        const uintptr_t as = (gs + 15) & ~static_cast<uintptr_t>(15), ae = ge & ~static_cast<uintptr_t>(15);
-        const uint32_t srow = scR0 + 4u * (((r - 1) & (kRing - 1)) * RS + static_cast<int>((gs >> 2) & 31));
-        int x0, x1;
-        if (t < CH) {
-          x0 = 0;
-          x1 = ae > as ? static_cast<int>((as - gs) >> 2) : ws;
-        } else {
-          x0 = ae > as ? static_cast<int>((ae - gs) >> 2) : ws;
-          x1 = ws;
-        }
-        for (int x = x0; x < x1; ++x) g[x] = lds_s32(srow + 4u * x);
+      const int r = static_cast<int>(row0) + i;
+      const uintptr_t gs = reinterpret_cast<uintptr_t>(Sb) + 4u * static_cast<uintptr_t>((row0 + i) * P.lds + c0);
+      const uintptr_t ge = gs + 4u * ws;
+      const uintptr_t as = (gs + 15) & ~static_cast<uintptr_t>(15), ae = ge & ~static_cast<uintptr_t>(15);
+      const uint32_t srow = scR0 + 4u * (((r - 1) & (kRing - 1)) * RS + static_cast<int>((gs >> 2) & 31));
+      const bool row_ok = t < 2 * CH && r <= n;
+      int x0, x1;
+      if (t < CH) {
+        x0 = 0;
+        x1 = ae > as ? static_cast<int>((as - gs) >> 2) : ws;
+      } else {
+        x0 = ae > as ? static_cast<int>((ae - gs) >> 2) : ws;
+        x1 = ws;
+      }
+      if (x1 - x0 <= 3) {
+        int hv[3];
+#pragma unroll
+        for (int x = 0; x < 3; ++x) hv[x] = lds32_p(row_ok && x0 + x < x1, srow + 4u * (x0 + x));
+#pragma unroll
+        for (int x = 0; x < 3; ++x) stg32_p(row_ok && x0 + x < x1, reinterpret_cast<void*>(gs + 4u * (x0 + x)), hv[x]);
+      } else if (row_ok) {  // narrow band (< 16 bytes of aligned interior): all words scalar
+        for (int x = x0; x < x1; ++x) stg32_p(true, reinterpret_cast<void*>(gs + 4u * x), lds_s32(srow + 4u * x));
       }
     }
   };
