@@ -278,80 +278,132 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
   };
 
   // Per-lane staging assignments, fixed for the whole task: in iteration it lane t moves the
-  // 16-byte chunk k of row i of a CH-row chunk (f = t + 32*it, i = f / MAX, k = f % MAX).
-  // Row addresses advance by CH*ld per chunk; with CH a multiple of 4 and ld odd the 16-byte
-  // phase of row i is the same in every chunk.
-  const char* const Rb = reinterpret_cast<const char*>(R);
-  char* const Sb = reinterpret_cast<char*>(S);
-  // ref chunk c (rows CH*c+1 .. CH*c+CH): straight-line predicated cp.async (LDGSTS), then every
-  // lane arrives on the chunk's mbarrier when its copies have landed.
-  auto issue_ref = [&](int c) {
-    const long long row0 = static_cast<long long>(c) * CH + 1;
+  // 16-byte chunk k of row i of a CH-row chunk (f = t + 32*it, i = f / MAX, k = f % MAX).  Chunk c
+  // is chunk 0 moved by c*CH rows: global addresses by c*CH*ld words, ring rows by c*CH, and the
+  // swizzle G & 31 by D_c = c*CH*ld mod 32; with CH a multiple of 4 the 16-byte phase of row i
+  // (G & 3) is the same in every chunk, so every per-lane offset below is precomputed once.
+  uintptr_t rsrc[C::ITER_R];  // chunk-0 source byte address (16-byte aligned)
+  uint32_t rdst[C::ITER_R];   // ring byte offset within a chunk: i*RS*4 + 16k
+  int rg[C::ITER_R];          // G(row i of chunk 0) & 31
+  bool rok[C::ITER_R];        // (row i, chunk k) exists for a full chunk
+  int rrow[C::ITER_R];        // i (row within chunk)
+  if constexpr (!SEQ) {
 #pragma unroll
     for (int it = 0; it < C::ITER_R; ++it) {
       const int f = t + 32 * it;
       const int i = f / C::MAXR, k = f - (f / C::MAXR) * C::MAXR;
-      const int r = static_cast<int>(row0) + i;
-      const uintptr_t gs = reinterpret_cast<uintptr_t>(Rb) + 4u * static_cast<uintptr_t>((row0 + i) * P.ldr + c0);
-      const uintptr_t ca = (gs & ~static_cast<uintptr_t>(15)) + 16u * k;
-      const uintptr_t e0 = (gs + 4u * ws + 15) & ~static_cast<uintptr_t>(15);
-      const uint32_t dst = refR0 + 4u * (((r - 1) & (kRing - 1)) * RS + static_cast<int>((gs >> 2) & 28)) + 16u * k;
-      const bool in = i < CH && r <= n && ca < e0;
-      cp_async16_p(in && ca + 16 <= rend, dst, reinterpret_cast<const void*>(ca));
-      if (in && ca + 16 > rend) {  // the matrix's last row: never read past its final element
-        for (int x = 0; x < 4; ++x)
-          if (ca + 4u * x < rend) cp_async4(dst + 4u * x, reinterpret_cast<const void*>(ca + 4u * x));
+      const uintptr_t G = GR0 + static_cast<uintptr_t>((1 + i) * P.ldr);
+      const int a = static_cast<int>(G & 3);
+      rsrc[it] = 4u * (G - a) + 16u * k;
+      rdst[it] = 4u * (i * RS) + 16u * k;
+      rg[it] = static_cast<int>(G & 31);
+      rok[it] = i < CH && 4 * k < a + ws;  // chunk k starts inside [G - a, align4(G + ws))
+      rrow[it] = i;
+    }
+  }
+  const uintptr_t rstride = 4u * static_cast<uintptr_t>(CH * P.ldr);
+  const int rDc = static_cast<int>((CH * P.ldr) & 31);
+  const int last_chunk = (n - 1) / CH;
+
+  // ref chunk c (rows CH*c+1 .. CH*c+CH): predicated cp.async (LDGSTS) from precomputed offsets,
+  // then every lane arrives on the chunk's mbarrier when its copies have landed.
+  auto issue_ref = [&](int c) {
+    const uintptr_t cb = static_cast<uintptr_t>(c) * rstride;
+    const uint32_t db = refR0 + 4u * ((c * CH) & (kRing - 1)) * RS;
+    const int Dc = (c * rDc) & 31;
+    const int rlim = n - c * CH;  // row i valid iff i < rlim
+    if (!(last_band && c == last_chunk)) {
+#pragma unroll
+      for (int it = 0; it < C::ITER_R; ++it) {
+        const uint32_t dst = db + rdst[it] + 4u * ((rg[it] + Dc) & 28);
+        cp_async16_p(rok[it] && rrow[it] < rlim, dst, reinterpret_cast<const void*>(rsrc[it] + cb));
+      }
+    } else {  // the matrix's last rows: never read past the final element
+#pragma unroll
+      for (int it = 0; it < C::ITER_R; ++it) {
+        const uint32_t dst = db + rdst[it] + 4u * ((rg[it] + Dc) & 28);
+        const uintptr_t ca = rsrc[it] + cb;
+        if (rok[it] && rrow[it] < rlim) {
+          if (ca + 16 <= rend) {
+            cp_async16(dst, reinterpret_cast<const void*>(ca));
+          } else {
+            for (int x = 0; x < 4; ++x)
+              if (ca + 4u * x < rend) cp_async4(dst + 4u * x, reinterpret_cast<const void*>(ca + 4u * x));
+          }
+        }
       }
     }
     cp_async_arrive(bar0 + 8 * (c % C::SLOTS));
   };
 
-  // score chunk c: all LDS.128 first, then all STG.128 (aligned interiors); scalar head/tail
-  // words (<= 3 each) by lanes 0..2CH-1
-  auto store_sc = [&](int c) {
-    const long long row0 = static_cast<long long>(c) * CH + 1;
-    int4 v[C::ITER_S];
-    uintptr_t dst[C::ITER_S];
-    bool ok[C::ITER_S];
+  // score stores, same scheme: interior 16-byte chunks (all LDS.128 first, then STG.128) and
+  // the <= 3 unaligned head (lanes 0..CH-1) / tail (lanes CH..2CH-1) words of each row
+  uintptr_t sdst[C::ITER_S];  // chunk-0 destination byte address (16-byte aligned)
+  uint32_t ssrc[C::ITER_S];   // ring byte offset within a chunk (without the swizzle)
+  int sg[C::ITER_S];          // G_S(row i of chunk 0) & 31
+  bool sok[C::ITER_S];
+  int srow_i[C::ITER_S];
 #pragma unroll
-    for (int it = 0; it < C::ITER_S; ++it) {
-      const int f = t + 32 * it;
-      const int i = f / C::MAXS, k = f - (f / C::MAXS) * C::MAXS;
-      const int r = static_cast<int>(row0) + i;
-      const uintptr_t gs = reinterpret_cast<uintptr_t>(Sb) + 4u * static_cast<uintptr_t>((row0 + i) * P.lds + c0);
-      const uintptr_t as = (gs + 15) & ~static_cast<uintptr_t>(15), ae = (gs + 4u * ws) & ~static_cast<uintptr_t>(15);
-      dst[it] = as + 16u * k;
-      ok[it] = i < CH && r <= n && dst[it] < ae;
-      const uint32_t srow = scR0 + 4u * (((r - 1) & (kRing - 1)) * RS + static_cast<int>((gs >> 2) & 31));
-      v[it] = lds128_p(ok[it], srow + static_cast<uint32_t>(dst[it] - gs));
+  for (int it = 0; it < C::ITER_S; ++it) {
+    const int f = t + 32 * it;
+    const int i = f / C::MAXS, k = f - (f / C::MAXS) * C::MAXS;
+    const uintptr_t G = GS0 + static_cast<uintptr_t>((1 + i) * P.lds);
+    const int a = static_cast<int>(G & 3);
+    const int h = (4 - a) & 3;                                   // unaligned head words
+    const int nint = ws > h ? (ws - h) >> 2 : 0;                 // aligned 16-byte chunks
+    sdst[it] = 4u * (G + h) + 16u * k;
+    ssrc[it] = 4u * (i * RS + h) + 16u * k;
+    sg[it] = static_cast<int>(G & 31);
+    sok[it] = i < CH && k < nint;
+    srow_i[it] = i;
+  }
+  // head / tail words of row ht_i = t % CH (lanes < 2CH)
+  int ht_x0, ht_x1;
+  uintptr_t ht_g;
+  int ht_gsw;
+  {
+    const int i = t % CH;
+    const uintptr_t G = GS0 + static_cast<uintptr_t>((1 + i) * P.lds);
+    const int a = static_cast<int>(G & 3);
+    const int h = min((4 - a) & 3, ws);
+    const int nint = ws > h ? (ws - h) >> 2 : 0;
+    if (t < CH) {
+      ht_x0 = 0;
+      ht_x1 = h;
+    } else {
+      ht_x0 = h + 4 * nint;
+      ht_x1 = t < 2 * CH ? ws : ht_x0;
     }
+    ht_g = 4u * G;
+    ht_gsw = static_cast<int>(G & 31);
+  }
+  const uintptr_t sstride = 4u * static_cast<uintptr_t>(CH * P.lds);
+  const int sDc = static_cast<int>((CH * P.lds) & 31);
+
+  auto store_sc = [&](int c) {
+    const uintptr_t cb = static_cast<uintptr_t>(c) * sstride;
+    const uint32_t sb = scR0 + 4u * ((c * CH) & (kRing - 1)) * RS;
+    const int Dc = (c * sDc) & 31;
+    const int rlim = n - c * CH;
+    int4 v[C::ITER_S];
 #pragma unroll
-    for (int it = 0; it < C::ITER_S; ++it) stg128_p(ok[it], reinterpret_cast<void*>(dst[it]), v[it]);
-    {  // lanes 0..CH-1: head words of row t; lanes CH..2CH-1: tail words of row t-CH
-      const int i = t % CH;
-      const int r = static_cast<int>(row0) + i;
-      const uintptr_t gs = reinterpret_cast<uintptr_t>(Sb) + 4u * static_cast<uintptr_t>((row0 + i) * P.lds + c0);
-      const uintptr_t ge = gs + 4u * ws;
-      const uintptr_t as = (gs + 15) & ~static_cast<uintptr_t>(15), ae = ge & ~static_cast<uintptr_t>(15);
-      const uint32_t srow = scR0 + 4u * (((r - 1) & (kRing - 1)) * RS + static_cast<int>((gs >> 2) & 31));
-      const bool row_ok = t < 2 * CH && r <= n;
-      int x0, x1;
-      if (t < CH) {
-        x0 = 0;
-        x1 = ae > as ? static_cast<int>((as - gs) >> 2) : ws;
-      } else {
-        x0 = ae > as ? static_cast<int>((ae - gs) >> 2) : ws;
-        x1 = ws;
-      }
-      if (x1 - x0 <= 3) {
-        int hv[3];
+    for (int it = 0; it < C::ITER_S; ++it)
+      v[it] = lds128_p(sok[it] && srow_i[it] < rlim, sb + ssrc[it] + 4u * ((sg[it] + Dc) & 31));
 #pragma unroll
-        for (int x = 0; x < 3; ++x) hv[x] = lds32_p(row_ok && x0 + x < x1, srow + 4u * (x0 + x));
+    for (int it = 0; it < C::ITER_S; ++it)
+      stg128_p(sok[it] && srow_i[it] < rlim, reinterpret_cast<void*>(sdst[it] + cb), v[it]);
+    // head / tail
+    const bool row_ok = (t % CH) < rlim;
+    const uint32_t hb = sb + 4u * ((t % CH) * RS + ((ht_gsw + Dc) & 31));
+    if (ht_x1 - ht_x0 <= 3) {
+      int hv[3];
 #pragma unroll
-        for (int x = 0; x < 3; ++x) stg32_p(row_ok && x0 + x < x1, reinterpret_cast<void*>(gs + 4u * (x0 + x)), hv[x]);
-      } else if (row_ok) {  // narrow band (< 16 bytes of aligned interior): all words scalar
-        for (int x = x0; x < x1; ++x) stg32_p(true, reinterpret_cast<void*>(gs + 4u * x), lds_s32(srow + 4u * x));
-      }
+      for (int x = 0; x < 3; ++x) hv[x] = lds32_p(row_ok && ht_x0 + x < ht_x1, hb + 4u * (ht_x0 + x));
+#pragma unroll
+      for (int x = 0; x < 3; ++x)
+        stg32_p(row_ok && ht_x0 + x < ht_x1, reinterpret_cast<void*>(ht_g + cb + 4u * (ht_x0 + x)), hv[x]);
+    } else if (row_ok) {  // narrow band (< 16 bytes of aligned interior): every word scalar
+      for (int x = ht_x0; x < ht_x1; ++x) stg32_p(true, reinterpret_cast<void*>(ht_g + cb + 4u * x), lds_s32(hb + 4u * x));
     }
   };
 
