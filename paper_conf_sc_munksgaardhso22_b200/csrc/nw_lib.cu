@@ -81,7 +81,7 @@ cudaError_t setup_kernel(int* occ) {
   cudaError_t e = cudaFuncSetAttribute(nw_strip_kernel<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        static_cast<int>(C::kSmem));
   if (e != cudaSuccess) return e;
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, nw_strip_kernel<C>, 32 * C::NW, C::kSmem);
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, nw_strip_kernel<C>, 64 * C::NW, C::kSmem);
 }
 
 std::mutex g_mu;
@@ -226,13 +226,13 @@ nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* 
   w->ticket_next += static_cast<unsigned long long>(P.ngroups + grid);  // every CTA draws one extra ticket
   const unsigned g = static_cast<unsigned>(grid);
   if (K == 2 && !SEQ)
-    nw_strip_kernel<CfgK2><<<g, 32 * CfgK2::NW, CfgK2::kSmem, st>>>(P);
+    nw_strip_kernel<CfgK2><<<g, 64 * CfgK2::NW, CfgK2::kSmem, st>>>(P);
   else if (K == 2)
-    nw_strip_kernel<CfgK2S><<<g, 32 * CfgK2S::NW, CfgK2S::kSmem, st>>>(P);
+    nw_strip_kernel<CfgK2S><<<g, 64 * CfgK2S::NW, CfgK2S::kSmem, st>>>(P);
   else if (!SEQ)
-    nw_strip_kernel<CfgK4><<<g, 32 * CfgK4::NW, CfgK4::kSmem, st>>>(P);
+    nw_strip_kernel<CfgK4><<<g, 64 * CfgK4::NW, CfgK4::kSmem, st>>>(P);
   else
-    nw_strip_kernel<CfgK4S><<<g, 32 * CfgK4S::NW, CfgK4S::kSmem, st>>>(P);
+    nw_strip_kernel<CfgK4S><<<g, 64 * CfgK4S::NW, CfgK4S::kSmem, st>>>(P);
   NW_CU(cudaGetLastError());
   return NW_OK;
 }

@@ -45,7 +45,7 @@
 
 namespace nwb200 {
 
-constexpr int kBarBytes = 128;
+constexpr int kBarBytes = 512;  // per band pair: ref_full[16], ev[16], st_done[16] mbarriers
 constexpr int kBR = 256;      // shared border ring entries between consecutive warps of a CTA
 constexpr int kRing = 64;     // rows per staging ring (power of two)
 constexpr unsigned kErrWatchdog = 0xBADB0001u;
@@ -76,6 +76,7 @@ struct StripCfg {
   static_assert(RS % 4 == 0 && kWarpSmem % 16 == 0, "16-byte aligned rings");
   static_assert(((size_t)kRing * RS) % 32 == 0, "ring wrap keeps banks");
   static_assert(NW <= 8 && SLOTS <= 16, "header / barrier space");
+  static constexpr int LOOKW = SLOTS - SKEW - 1;     // ref chunks the staging warp runs ahead
 };
 
 // ---- the schedule (shared by the kernel and the host export nw_strip_map, pin P7) --------
@@ -189,7 +190,7 @@ enum : int { kSinkNone = 0, kSinkSmem = 1, kSinkGlobal = 2 };
 template <class C, int SINK>
 __device__ __forceinline__ void nw_band(const StripParams& P, const long long task, const int w, const int t,
                                         unsigned char* const smem, unsigned char* const wsm, const uint32_t gen,
-                                        uint32_t& ph) {
+                                        uint32_t& ph_rf, uint32_t& ph_sd) {
   constexpr int K = C::K, RS = C::RS, CH = C::CH;
   constexpr bool SEQ = C::SEQ;
   constexpr unsigned FULL = 0xffffffffu;
@@ -197,11 +198,10 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
   const long long c_task0 = clock64();
   const bool tracing = P.trace != nullptr;
   long long ev_cyc = 0, spin_cyc = 0, wait_cyc = 0;  // debug cycle accounting (trace only)
-  long long st_cyc = 0, is_cyc = 0;
 
   const uint32_t s_prog = smem_u32(smem + 8);
   const uint32_t s_bring = smem_u32(smem + 128);
-  const uint32_t bar0 = smem_u32(wsm);
+  const uint32_t bar_rf = smem_u32(wsm), bar_ev = bar_rf + 128, bar_sd = bar_rf + 256;
   int32_t* const ref_ring = reinterpret_cast<int32_t*>(wsm + kBarBytes);
   int32_t* const sc_ring = ref_ring + C::REF_ROWS * RS;
   uint32_t* const prof = reinterpret_cast<uint32_t*>(sc_ring + kRing * RS);
@@ -276,6 +276,227 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
     if (src == kSrcSmem) return hi == (gen | static_cast<uint32_t>(row));
     return true;
   };
+
+  // ---- prologue: top border (row 0 is input), left-border window, first ref chunks
+  int Pv[K];
+#pragma unroll
+  for (int m = 0; m < K; ++m) Pv[m] = (t * K + m < ws) ? __ldg(S + c0 + t * K + m) : 0;
+  int Lprev = (t * K < ws) ? __ldg(S + c0 + t * K - 1) : 0;  // diag input of the first row
+  int vlast = Pv[K - 1];
+  int win_base = 1;  // cur holds border rows win_base + t
+  uint64_t cur = load_entry(1 + t);
+  uint64_t nxt = src == kSrcSmem ? 0ull : load_entry(33 + t);
+  // per-lane ring addressing: row r (= step + 1 - t) lives at ring row (r-1) & 63
+  const int r0 = 1 - t;
+  int rr = r0 - 1;  // r - 1
+  int gR = static_cast<int>((GR0 + static_cast<uintptr_t>(static_cast<intptr_t>(r0) * P.ldr)) & 31);
+  int gS = static_cast<int>((GS0 + static_cast<uintptr_t>(static_cast<intptr_t>(r0) * P.lds)) & 31);
+  const int ldr32 = static_cast<int>(P.ldr & 31), lds32 = static_cast<int>(P.lds & 31);
+  const uint32_t laneR = refR0 + 4u * t * K, laneS = scR0 + 4u * t * K;
+  // right-border publish (lane out_lane holds the band's last column in Pv[K-1]; every band
+  // with a right neighbour is full width)
+  const bool do_out = t == out_lane;
+  uint64_t* gout = lout != nullptr ? lout + r0 : nullptr;
+  uint32_t sout_hi = lout_tag + static_cast<uint32_t>(r0);
+  // SEQ: per-band substitution profile prof[x][t] = pack_m subst[x][b[c0-1+tK+m]] (int8 x K)
+  const uint8_t* const A = SEQ ? P.seq_a + pair * P.psa : nullptr;
+  int a0 = 0, a1 = 0;  // residues of this lane's current and next row (software pipeline)
+  if constexpr (SEQ) {
+    const uint8_t* const Bq = P.seq_b + pair * P.psb;
+    int bj[K];
+#pragma unroll
+    for (int m = 0; m < K; ++m) bj[m] = (t * K + m < ws) ? (Bq[c0 - 1 + t * K + m] & 31) : 0;
+    for (int x = 0; x < 32; ++x) {
+      uint32_t wv = 0;
+#pragma unroll
+      for (int m = 0; m < K; ++m)
+        wv |= static_cast<uint32_t>(static_cast<uint8_t>(P.subst[x * 32 + bj[m]])) << (8 * m);
+      prof[x * 32 + t] = wv;
+    }
+    a0 = A[min(max(r0 - 1, 0), n - 1)] & 31;
+    a1 = A[min(max(r0, 0), n - 1)] & 31;
+    __syncwarp();
+  }
+  const uint32_t* const profp = prof + t;
+  uint32_t tok = 0;  // produced by each chunk's mbarrier wait, consumed by the ref loads
+
+  // one wavefront step; ALL = every lane's row is in 1..n (steady state, no predicates)
+  auto step = [&](const int sig, auto all_tag) {
+    constexpr bool ALL = decltype(all_tag)::value;
+    const uint32_t roff = 4u * RS * static_cast<uint32_t>(rr & (kRing - 1));
+    int rv[K];
+    if constexpr (SEQ) {
+      const uint32_t pw = profp[32 * a0];
+#pragma unroll
+      for (int m = 0; m < K; ++m) rv[m] = prmt_sext(pw, 0x8880u + 0x1111u * m);  // sign-extended byte m
+    } else {
+      const uint32_t aR = laneR + roff + 4u * static_cast<uint32_t>(gR & 31);
+#pragma unroll
+      for (int m = 0; m < K; ++m) rv[m] = lds_tok(aR + 4 * m, tok);
+    }
+    const int bval = __shfl_sync(FULL, static_cast<int>(static_cast<uint32_t>(cur)), sig & 31);
+    const int from_left = __shfl_up_sync(FULL, vlast, 1);
+    const int L = (t == 0) ? bval : from_left;
+    bool active = true;
+    if (!ALL) {
+      const int r = lane_row(sig, t);
+      active = r >= 1 && r <= n;
+    }
+    if (active) {
+      int d = Lprev, l = L;
+#pragma unroll
+      for (int m = 0; m < K; ++m) {
+        const int x = __viaddmax_s32(Pv[m], -p, d + rv[m]);  // max(up - p, diag + ref)
+        const int v = __viaddmax_s32(l, -p, x);              // max(left - p, .)
+        d = Pv[m];
+        Pv[m] = v;
+        l = v;
+      }
+      Lprev = L;
+      const uint32_t aS = laneS + roff + 4u * static_cast<uint32_t>(gS & 31);
+#pragma unroll
+      for (int m = 0; m < K; ++m) sts_s32(aS + 4 * m, Pv[m]);
+      const uint32_t vo = static_cast<uint32_t>(Pv[K - 1]);
+      if constexpr (SINK == kSinkSmem) {
+        st_entry_smem(do_out, bring_out + 8u * (sout_hi & (kBR - 1)), vo, sout_hi);
+      } else if constexpr (SINK == kSinkGlobal) {
+        st_entry_gpu(do_out && !lout_sys, gout, vo, lout_tag);
+        st_entry_sys(do_out && lout_sys, gout, vo, lout_tag);
+      } else {
+        (void)vo;
+      }
+    }
+    vlast = Pv[K - 1];
+    // advance this lane to row r+1
+    if constexpr (SEQ) {
+      a0 = a1;
+      a1 = __ldg(A + min(max(lane_row(sig, t) + 1, 0), n - 1)) & 31;  // residue of row r+2
+    }
+    ++rr;
+    gR += ldr32;
+    gS += lds32;
+    if constexpr (SINK == kSinkGlobal) ++gout;
+    if constexpr (SINK == kSinkSmem) ++sout_hi;
+  };
+
+  for (int Q = 0; Q <= nch + C::STORE_DELAY - 1; ++Q) {
+    const int sig0 = Q * CH;
+    const long long c_ev0 = tracing ? clock64() : 0;
+    // ---- chunk events (warp-uniform).  The paired staging warp stores finished score chunks
+    // and prefetches ref chunks; this warp only synchronises with it.
+    if (Q < nch) {
+      const long long c_w0 = tracing ? clock64() : 0;
+      const int sl = Q % C::SLOTS;
+      if (Q >= C::SLOTS) {  // score slot of chunk Q is free once chunk Q-SLOTS was stored
+        mbar_wait(bar_sd + 8 * sl, (ph_sd >> sl) & 1u);
+        ph_sd ^= 1u << sl;
+      }
+      if constexpr (!SEQ) {
+        tok = mbar_wait_tok(bar_rf + 8 * sl, (ph_rf >> sl) & 1u);
+        ph_rf ^= 1u << sl;
+      }
+      if (tracing) wait_cyc += clock64() - c_w0;
+    }
+    // event Q reached: score chunk Q-STORE_DELAY is complete, ref chunk Q-SKEW-1 no longer read
+    __syncwarp();
+    if (t == 0) mbar_arrive(bar_ev + 8 * (Q % C::SLOTS));
+    if (sig0 >= nsteps) {
+      if (tracing) ev_cyc += clock64() - c_ev0;
+      continue;
+    }
+    if (src == kSrcSmem && t == 0) sts32_volatile(prog_in, sig0);  // rows <= sig0 consumed
+    if ((sig0 & 31) == 0 && sig0 > 0) {
+      cur = src == kSrcSmem ? load_entry(sig0 + 1 + t) : nxt;
+      win_base = sig0 + 1;
+      if (src != kSrcSmem) nxt = load_entry(sig0 + 33 + t);
+    }
+    if (src != kSrcPlain) {
+      // the block needs rows sig0+1 .. sig0+CH of the left border (lanes j0 .. j0+CH-1)
+      const int j0 = sig0 & 31;
+      auto ready = [&]() {
+        const int row = win_base + t;
+        const bool need = t >= j0 && t < j0 + CH && row <= n;
+        return __all_sync(FULL, !need || entry_ok(cur, row)) != 0;
+      };
+      if (!ready()) {
+        const long long c_0 = clock64();
+        const uint64_t t0 = globaltimer_ns();
+        unsigned spins = 0;
+        do {
+          cur = load_entry(win_base + t);
+          if ((++spins & 255u) == 0 && globaltimer_ns() - t0 > P.spin_limit_ns) watchdog_trap(P.err);
+        } while (!ready());
+        spin_cyc += clock64() - c_0;
+      }
+    }
+    if constexpr (SINK == kSinkSmem) {
+      // back-pressure: rows written in this block are <= sig0+CH-31; their ring slots must hold
+      // rows the consumer (warp w+1) already consumed
+      const int rmax = sig0 + CH - 31;
+      if (rmax - kBR > 0 && rmax - kBR > lds32_volatile(prog_out)) {
+        const uint64_t t0 = globaltimer_ns();
+        while (rmax - kBR > lds32_volatile(prog_out))
+          if (globaltimer_ns() - t0 > P.spin_limit_ns) watchdog_trap(P.err);
+      }
+    }
+    if (tracing) ev_cyc += clock64() - c_ev0;
+    // ---- CH wavefront steps: lane t computes row sig+1-t, columns c0+tK .. c0+tK+K-1
+    if (sig0 >= 31 && sig0 + CH <= n) {  // steady state: all 32 lanes on rows 1..n
+#pragma unroll
+      for (int j = 0; j < CH; ++j) step(sig0 + j, std::true_type{});
+    } else {
+#pragma unroll 1
+      for (int j = 0; j < CH; ++j) {
+        if (sig0 + j >= nsteps) break;
+        step(sig0 + j, std::false_type{});
+      }
+    }
+  }
+  __syncwarp();
+  if (P.trace != nullptr && t == 0 && task < P.trace_cap) {
+    unsigned smid;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+    unsigned long long* e = P.trace + 8 * task;
+    e[0] = static_cast<unsigned long long>(task);
+    e[1] = t_task0;
+    e[2] = globaltimer_ns();
+    e[3] = smid;
+    e[4] = static_cast<unsigned long long>(ev_cyc);    // cycles in chunk events (incl. waits)
+    e[5] = static_cast<unsigned long long>(wait_cyc);  // of which: waits on the staging warp
+    e[6] = static_cast<unsigned long long>(spin_cyc);  // of which: left-border spins
+    e[7] = static_cast<unsigned long long>(clock64() - c_task0);
+  }
+}
+
+
+// The staging warp paired with a compute warp: prefetches ref chunks (LOOKW ahead) and stores
+// finished score chunks, driven by the compute warp's per-event mbarrier arrivals.
+template <class C>
+__device__ __forceinline__ void nw_stage(const StripParams& P, const long long task, const int t,
+                                         unsigned char* const wsm, uint32_t& ph_ev) {
+  constexpr int RS = C::RS, CH = C::CH;
+  constexpr bool SEQ = C::SEQ;
+  const long long c_task0 = clock64();
+  long long wait_cyc = 0;
+  const uint32_t bar_rf = smem_u32(wsm), bar_ev = bar_rf + 128, bar_sd = bar_rf + 256;
+  int32_t* const ref_ring = reinterpret_cast<int32_t*>(wsm + kBarBytes);
+  int32_t* const sc_ring = ref_ring + C::REF_ROWS * RS;
+  const int n = static_cast<int>(P.n);
+  const int nch = (n + CH - 1) / CH;
+  const long long pair = task / P.nbands;
+  const int band = static_cast<int>(task - pair * P.nbands);
+  const bool last_band = band == P.nbands - 1;
+  const int c0 = band_c0(band, C::W);
+  const int ws = band_ws(P.width, band, C::W);
+  int32_t* const S = P.score + pair * P.pss;
+  const int32_t* const R = SEQ ? nullptr : P.ref + pair * P.psr;
+  const uintptr_t GR0 = SEQ ? 0 : (reinterpret_cast<uintptr_t>(R) >> 2) + c0;  // word addr of (0, c0)
+  const uintptr_t GS0 = (reinterpret_cast<uintptr_t>(S) >> 2) + c0;
+  const uintptr_t rend =
+      SEQ ? 0 : reinterpret_cast<uintptr_t>(R + static_cast<long long>(n) * P.ldr + P.width + 1);  // past the last element
+  const uint32_t refR0 = opaque(smem_u32(ref_ring));
+  const uint32_t scR0 = opaque(smem_u32(sc_ring));
+  const uint32_t bar0 = bar_rf;
 
   // Per-lane staging assignments, fixed for the whole task: in iteration it lane t moves the
   // 16-byte chunk k of row i of a CH-row chunk (f = t + 32*it, i = f / MAX, k = f % MAX).  Chunk c
@@ -407,224 +628,59 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
     }
   };
 
-  // ---- prologue: top border (row 0 is input), left-border window, first ref chunks
-  int Pv[K];
-#pragma unroll
-  for (int m = 0; m < K; ++m) Pv[m] = (t * K + m < ws) ? __ldg(S + c0 + t * K + m) : 0;
-  int Lprev = (t * K < ws) ? __ldg(S + c0 + t * K - 1) : 0;  // diag input of the first row
-  int vlast = Pv[K - 1];
-  int win_base = 1;  // cur holds border rows win_base + t
-  uint64_t cur = load_entry(1 + t);
-  uint64_t nxt = src == kSrcSmem ? 0ull : load_entry(33 + t);
-  // per-lane ring addressing: row r (= step + 1 - t) lives at ring row (r-1) & 63
-  const int r0 = 1 - t;
-  int rr = r0 - 1;  // r - 1
-  int gR = static_cast<int>((GR0 + static_cast<uintptr_t>(static_cast<intptr_t>(r0) * P.ldr)) & 31);
-  int gS = static_cast<int>((GS0 + static_cast<uintptr_t>(static_cast<intptr_t>(r0) * P.lds)) & 31);
-  const int ldr32 = static_cast<int>(P.ldr & 31), lds32 = static_cast<int>(P.lds & 31);
-  const uint32_t laneR = refR0 + 4u * t * K, laneS = scR0 + 4u * t * K;
-  // right-border publish (lane out_lane holds the band's last column in Pv[K-1]; every band
-  // with a right neighbour is full width)
-  const bool do_out = t == out_lane;
-  uint64_t* gout = lout != nullptr ? lout + r0 : nullptr;
-  uint32_t sout_hi = lout_tag + static_cast<uint32_t>(r0);
   if constexpr (!SEQ) {
-    for (int c = 0; c < C::LOOK && c < nch; ++c) issue_ref(c);
+    for (int c = 0; c < C::LOOKW && c < nch; ++c) issue_ref(c);
   }
-  // SEQ: per-band substitution profile prof[x][t] = pack_m subst[x][b[c0-1+tK+m]] (int8 x K)
-  const uint8_t* const A = SEQ ? P.seq_a + pair * P.psa : nullptr;
-  int a0 = 0, a1 = 0;  // residues of this lane's current and next row (software pipeline)
-  if constexpr (SEQ) {
-    const uint8_t* const Bq = P.seq_b + pair * P.psb;
-    int bj[K];
-#pragma unroll
-    for (int m = 0; m < K; ++m) bj[m] = (t * K + m < ws) ? (Bq[c0 - 1 + t * K + m] & 31) : 0;
-    for (int x = 0; x < 32; ++x) {
-      uint32_t wv = 0;
-#pragma unroll
-      for (int m = 0; m < K; ++m)
-        wv |= static_cast<uint32_t>(static_cast<uint8_t>(P.subst[x * 32 + bj[m]])) << (8 * m);
-      prof[x * 32 + t] = wv;
-    }
-    a0 = A[min(max(r0 - 1, 0), n - 1)] & 31;
-    a1 = A[min(max(r0, 0), n - 1)] & 31;
-    __syncwarp();
-  }
-  const uint32_t* const profp = prof + t;
-  uint32_t tok = 0;  // produced by each chunk's mbarrier wait, consumed by the ref loads
-
-  // one wavefront step; ALL = every lane's row is in 1..n (steady state, no predicates)
-  auto step = [&](const int sig, auto all_tag) {
-    constexpr bool ALL = decltype(all_tag)::value;
-    const uint32_t roff = 4u * RS * static_cast<uint32_t>(rr & (kRing - 1));
-    int rv[K];
-    if constexpr (SEQ) {
-      const uint32_t pw = profp[32 * a0];
-#pragma unroll
-      for (int m = 0; m < K; ++m) rv[m] = prmt_sext(pw, 0x8880u + 0x1111u * m);  // sign-extended byte m
-    } else {
-      const uint32_t aR = laneR + roff + 4u * static_cast<uint32_t>(gR & 31);
-#pragma unroll
-      for (int m = 0; m < K; ++m) rv[m] = lds_tok(aR + 4 * m, tok);
-    }
-    const int bval = __shfl_sync(FULL, static_cast<int>(static_cast<uint32_t>(cur)), sig & 31);
-    const int from_left = __shfl_up_sync(FULL, vlast, 1);
-    const int L = (t == 0) ? bval : from_left;
-    bool active = true;
-    if (!ALL) {
-      const int r = lane_row(sig, t);
-      active = r >= 1 && r <= n;
-    }
-    if (active) {
-      int d = Lprev, l = L;
-#pragma unroll
-      for (int m = 0; m < K; ++m) {
-        const int x = __viaddmax_s32(Pv[m], -p, d + rv[m]);  // max(up - p, diag + ref)
-        const int v = __viaddmax_s32(l, -p, x);              // max(left - p, .)
-        d = Pv[m];
-        Pv[m] = v;
-        l = v;
-      }
-      Lprev = L;
-      const uint32_t aS = laneS + roff + 4u * static_cast<uint32_t>(gS & 31);
-#pragma unroll
-      for (int m = 0; m < K; ++m) sts_s32(aS + 4 * m, Pv[m]);
-      const uint32_t vo = static_cast<uint32_t>(Pv[K - 1]);
-      if constexpr (SINK == kSinkSmem) {
-        st_entry_smem(do_out, bring_out + 8u * (sout_hi & (kBR - 1)), vo, sout_hi);
-      } else if constexpr (SINK == kSinkGlobal) {
-        st_entry_gpu(do_out && !lout_sys, gout, vo, lout_tag);
-        st_entry_sys(do_out && lout_sys, gout, vo, lout_tag);
-      } else {
-        (void)vo;
-      }
-    }
-    vlast = Pv[K - 1];
-    // advance this lane to row r+1
-    if constexpr (SEQ) {
-      a0 = a1;
-      a1 = __ldg(A + min(max(lane_row(sig, t) + 1, 0), n - 1)) & 31;  // residue of row r+2
-    }
-    ++rr;
-    gR += ldr32;
-    gS += lds32;
-    if constexpr (SINK == kSinkGlobal) ++gout;
-    if constexpr (SINK == kSinkSmem) ++sout_hi;
-  };
-
   for (int Q = 0; Q <= nch + C::STORE_DELAY - 1; ++Q) {
-    const int sig0 = Q * CH;
-    const long long c_ev0 = tracing ? clock64() : 0;
-    // ---- chunk events (warp-uniform)
-    if (Q >= C::STORE_DELAY && Q - C::STORE_DELAY < nch) store_sc(Q - C::STORE_DELAY);
-    const long long c_st1 = tracing ? clock64() : 0;
-    if (tracing) st_cyc += c_st1 - c_ev0;
+    const int sl = Q % C::SLOTS;
+    const long long c_w0 = clock64();
+    mbar_wait(bar_ev + 8 * sl, (ph_ev >> sl) & 1u);
+    ph_ev ^= 1u << sl;
+    wait_cyc += clock64() - c_w0;
+    const int cs = Q - C::STORE_DELAY;
+    if (cs >= 0 && cs < nch) {
+      store_sc(cs);
+      __syncwarp();
+      if (t == 0) mbar_arrive(bar_sd + 8 * (cs % C::SLOTS));
+    }
     if constexpr (!SEQ) {
-      if (Q + C::LOOK < nch) issue_ref(Q + C::LOOK);
-      if (tracing) is_cyc += clock64() - c_st1;
-      if (Q < nch) {
-        const long long c_w0 = tracing ? clock64() : 0;
-        const int sl = Q % C::SLOTS;
-        tok = mbar_wait_tok(bar0 + 8 * sl, (ph >> sl) & 1u);
-        ph ^= 1u << sl;
-        if (tracing) wait_cyc += clock64() - c_w0;
-      }
-    }
-    __syncwarp();  // chunk copies / stored rows are settled for every lane
-    if (sig0 >= nsteps) {
-      if (tracing) ev_cyc += clock64() - c_ev0;
-      continue;
-    }
-    if (src == kSrcSmem && t == 0) sts32_volatile(prog_in, sig0);  // rows <= sig0 consumed
-    if ((sig0 & 31) == 0 && sig0 > 0) {
-      cur = src == kSrcSmem ? load_entry(sig0 + 1 + t) : nxt;
-      win_base = sig0 + 1;
-      if (src != kSrcSmem) nxt = load_entry(sig0 + 33 + t);
-    }
-    if (src != kSrcPlain) {
-      // the block needs rows sig0+1 .. sig0+CH of the left border (lanes j0 .. j0+CH-1)
-      const int j0 = sig0 & 31;
-      auto ready = [&]() {
-        const int row = win_base + t;
-        const bool need = t >= j0 && t < j0 + CH && row <= n;
-        return __all_sync(FULL, !need || entry_ok(cur, row)) != 0;
-      };
-      if (!ready()) {
-        const long long c_0 = clock64();
-        const uint64_t t0 = globaltimer_ns();
-        unsigned spins = 0;
-        do {
-          cur = load_entry(win_base + t);
-          if ((++spins & 255u) == 0 && globaltimer_ns() - t0 > P.spin_limit_ns) watchdog_trap(P.err);
-        } while (!ready());
-        spin_cyc += clock64() - c_0;
-      }
-    }
-    if constexpr (SINK == kSinkSmem) {
-      // back-pressure: rows written in this block are <= sig0+CH-31; their ring slots must hold
-      // rows the consumer (warp w+1) already consumed
-      const int rmax = sig0 + CH - 31;
-      if (rmax - kBR > 0 && rmax - kBR > lds32_volatile(prog_out)) {
-        const uint64_t t0 = globaltimer_ns();
-        while (rmax - kBR > lds32_volatile(prog_out))
-          if (globaltimer_ns() - t0 > P.spin_limit_ns) watchdog_trap(P.err);
-      }
-    }
-    if (tracing) ev_cyc += clock64() - c_ev0;
-    // ---- CH wavefront steps: lane t computes row sig+1-t, columns c0+tK .. c0+tK+K-1
-    if (sig0 >= 31 && sig0 + CH <= n) {  // steady state: all 32 lanes on rows 1..n
-#pragma unroll
-      for (int j = 0; j < CH; ++j) step(sig0 + j, std::true_type{});
-    } else {
-#pragma unroll 1
-      for (int j = 0; j < CH; ++j) {
-        if (sig0 + j >= nsteps) break;
-        step(sig0 + j, std::false_type{});
-      }
+      if (Q + C::LOOKW < nch) issue_ref(Q + C::LOOKW);
     }
   }
-  __syncwarp();
-  if (P.trace != nullptr && t == 0 && task < P.trace_cap) {
-    unsigned smid;
-    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
-    unsigned long long* e = P.trace + 8 * task;
-    e[0] = static_cast<unsigned long long>(task);
-    e[1] = t_task0;
-    e[2] = globaltimer_ns();
-    e[3] = smid;
-    e[4] = static_cast<unsigned long long>(ev_cyc);    // cycles in chunk events (incl. waits)
-    e[5] = static_cast<unsigned long long>(wait_cyc);  // of which: ref mbarrier waits
-    e[6] = static_cast<unsigned long long>(spin_cyc);  // of which: left-border spins
-    e[7] = static_cast<unsigned long long>(clock64() - c_task0);
-    if (P.trace_cap < 0) return;
-  }
-  if (P.trace != nullptr && t == 0 && task < P.trace_cap && P.trace2 != nullptr) {
-    P.trace2[2 * task] = static_cast<unsigned long long>(st_cyc);
-    P.trace2[2 * task + 1] = static_cast<unsigned long long>(is_cyc);
+  if (P.trace2 != nullptr && t == 0 && task < P.trace_cap) {
+    P.trace2[2 * task] = static_cast<unsigned long long>(clock64() - c_task0);
+    P.trace2[2 * task + 1] = static_cast<unsigned long long>(wait_cyc);
   }
 }
 
 template <class C>
-__global__ void __launch_bounds__(32 * C::NW, 1) nw_strip_kernel(const __grid_constant__ StripParams P) {
+__global__ void __launch_bounds__(64 * C::NW, 1) nw_strip_kernel(const __grid_constant__ StripParams P) {
   constexpr int NW = C::NW;
   extern __shared__ __align__(128) unsigned char smem[];
   const int t = threadIdx.x & 31;
-  const int w = threadIdx.x >> 5;
+  const int wa = threadIdx.x >> 5;           // 0..NW-1 compute warps, NW..2NW-1 staging warps
+  const bool staging = wa >= NW;
+  const int w = staging ? wa - NW : wa;      // the band slot this warp serves
   // CTA header: [0] group ticket, [8 + 4w] consumer progress of warp w, [128..] border rings
   unsigned long long* const s_group = reinterpret_cast<unsigned long long*>(smem);
   const uint32_t s_prog = smem_u32(smem + 8);
   unsigned char* const wsm = smem + C::kCtaHdr + w * C::kWarpSmem;
-  if (t == 0 && !C::SEQ) {
-    for (int i = 0; i < C::SLOTS; ++i) mbar_init(smem_u32(wsm) + 8 * i, 32);
+  if (!staging && t == 0) {
+    const uint32_t b = smem_u32(wsm);
+    for (int i = 0; i < C::SLOTS; ++i) {
+      mbar_init(b + 8 * i, 32);        // ref_full: one cp.async arrival per staging lane
+      mbar_init(b + 128 + 8 * i, 1);   // ev: the compute warp reached an event
+      mbar_init(b + 256 + 8 * i, 1);   // st_done: the staging warp stored a score chunk
+    }
   }
   fence_mbar_init();
   // shared border rings start invalid (tag 0xFFFFFFFF never equals gen | row, row < 2^30)
-  for (int i = threadIdx.x; i < (NW - 1) * kBR; i += 32 * NW) reinterpret_cast<unsigned long long*>(smem + 128)[i] = ~0ull;
+  for (int i = threadIdx.x; i < (NW - 1) * kBR; i += 64 * NW) reinterpret_cast<unsigned long long*>(smem + 128)[i] = ~0ull;
   if (threadIdx.x < NW) sts32_volatile(s_prog + 4 * threadIdx.x, 0);
   __syncthreads();
 
-  uint32_t ph = 0;  // mbarrier phase bits of this warp's ref slots
-  int gcount = 0;   // groups processed by this CTA (generation of the shared border tags)
+  uint32_t ph_a = 0, ph_b = 0;  // mbarrier phase bits this warp waits on
+  int gcount = 0;               // groups processed by this CTA (generation of the shared border tags)
   for (;;) {
     if (threadIdx.x == 0) *s_group = atomicAdd(P.ticket, 1ull);
     __syncthreads();
@@ -633,22 +689,26 @@ __global__ void __launch_bounds__(32 * C::NW, 1) nw_strip_kernel(const __grid_co
     const long long task = group * NW + w;
     const uint32_t gen = static_cast<uint32_t>(gcount & 3) << 30;
     if (task < P.ntasks) {
-      const int band = static_cast<int>(task % P.nbands);
-      const bool last_band = band == P.nbands - 1;
-      int sink;
-      if (last_band)
-        sink = P.halo_out ? kSinkGlobal : kSinkNone;
-      else
-        sink = (w < NW - 1) ? kSinkSmem : kSinkGlobal;
-      if (sink == kSinkSmem)
-        nw_band<C, kSinkSmem>(P, task, w, t, smem, wsm, gen, ph);
-      else if (sink == kSinkGlobal)
-        nw_band<C, kSinkGlobal>(P, task, w, t, smem, wsm, gen, ph);
-      else
-        nw_band<C, kSinkNone>(P, task, w, t, smem, wsm, gen, ph);
+      if (staging) {
+        nw_stage<C>(P, task, t, wsm, ph_a);
+      } else {
+        const int band = static_cast<int>(task % P.nbands);
+        const bool last_band = band == P.nbands - 1;
+        int sink;
+        if (last_band)
+          sink = P.halo_out ? kSinkGlobal : kSinkNone;
+        else
+          sink = (w < NW - 1) ? kSinkSmem : kSinkGlobal;
+        if (sink == kSinkSmem)
+          nw_band<C, kSinkSmem>(P, task, w, t, smem, wsm, gen, ph_a, ph_b);
+        else if (sink == kSinkGlobal)
+          nw_band<C, kSinkGlobal>(P, task, w, t, smem, wsm, gen, ph_a, ph_b);
+        else
+          nw_band<C, kSinkNone>(P, task, w, t, smem, wsm, gen, ph_a, ph_b);
+      }
     }
     __syncthreads();  // group end: every warp done (shared border rings / progress reusable)
-    if (t == 0) sts32_volatile(s_prog + 4 * w, 0);  // ordered before the next group by its barrier
+    if (!staging && t == 0) sts32_volatile(s_prog + 4 * w, 0);  // ordered before the next group
     ++gcount;
   }
 }

@@ -33,7 +33,7 @@ def main(path, n=None):
         tot = t[:, 7].astype(float)
         cols = [("events", 4), ("ref waits", 5), ("border spins", 6)]
         if t.shape[1] >= 10:
-            cols += [("score stores", 8), ("ref issue", 9)]
+            cols += [("staging busy", 8), ("staging wait", 9)]
         for name, col in cols:
             fr = t[:, col] / np.maximum(tot, 1)
             print(f"  {name:13s}: mean {fr.mean()*100:5.1f}% of task cycles (band0 {fr[0]*100:5.1f}%)")
