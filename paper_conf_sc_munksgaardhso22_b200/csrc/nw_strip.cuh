@@ -452,6 +452,13 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
       }
     }
   }
+  // consume the staging warp's remaining "stored" arrivals (chunks nch-SLOTS .. nch-1) so the
+  // st_done phases stay in step across tasks
+  for (int c = max(0, nch - C::SLOTS); c < nch; ++c) {
+    const int sl = c % C::SLOTS;
+    mbar_wait(bar_sd + 8 * sl, (ph_sd >> sl) & 1u);
+    ph_sd ^= 1u << sl;
+  }
   __syncwarp();
   if (P.trace != nullptr && t == 0 && task < P.trace_cap) {
     unsigned smid;
