@@ -319,6 +319,9 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
   }
   const uint32_t* const profp = prof + t;
   uint32_t tok = 0;  // produced by each chunk's mbarrier wait, consumed by the ref loads
+  int negp[K];       // -(m+1) p
+#pragma unroll
+  for (int m = 0; m < K; ++m) negp[m] = -(m + 1) * p;
 
   // one wavefront step; ALL = every lane's row is in 1..n (steady state, no predicates)
   auto step = [&](const int sig, auto all_tag) {
@@ -343,15 +346,23 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
       active = r >= 1 && r <= n;
     }
     if (active) {
-      int d = Lprev, l = L;
+      // Lane-local max-plus prefix form of the K-cell row segment:
+      //   x_m = max(up_m - p, diag_m + ref_m),  Y_m = max(Y_{m-1} - p, x_m),
+      //   v_m = max(Y_m, L - (m+1) p)  ==  max(x_m, v_{m-1} - p) with v_{-1} = L.
+      // x and Y need only the row above, so the left value L (one shuffle away) enters the
+      // step's critical path through a single VIADDMNMX per cell.
+      int Y[K];
+      {
+        int d = Lprev;
 #pragma unroll
-      for (int m = 0; m < K; ++m) {
-        const int x = __viaddmax_s32(Pv[m], -p, d + rv[m]);  // max(up - p, diag + ref)
-        const int v = __viaddmax_s32(l, -p, x);              // max(left - p, .)
-        d = Pv[m];
-        Pv[m] = v;
-        l = v;
+        for (int m = 0; m < K; ++m) {
+          const int x = __viaddmax_s32(Pv[m], -p, d + rv[m]);  // max(up - p, diag + ref)
+          Y[m] = m == 0 ? x : __viaddmax_s32(Y[m - 1], -p, x);
+          d = Pv[m];
+        }
       }
+#pragma unroll
+      for (int m = 0; m < K; ++m) Pv[m] = __viaddmax_s32(L, negp[m], Y[m]);  // max(L - (m+1)p, Y_m)
       Lprev = L;
       const uint32_t aS = laneS + roff + 4u * static_cast<uint32_t>(gS & 31);
 #pragma unroll
