@@ -323,6 +323,24 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
 #pragma unroll
   for (int m = 0; m < K; ++m) negp[m] = -(m + 1) * p;
 
+  // ref values are software-pipelined one step ahead: rvn holds row r's values when step s
+  // (row r) starts, and the loads for row r+1 are issued before the step's arithmetic, so the
+  // LDS latency hides behind the step's shuffle chain.
+  int rvn[K];
+  auto load_ref = [&](int out[K], int rr_, int gR_) {
+    if constexpr (SEQ) {
+      (void)rr_;
+      (void)gR_;
+    } else {
+      const uint32_t aR = laneR + 4u * RS * static_cast<uint32_t>(rr_ & (kRing - 1)) + 4u * static_cast<uint32_t>(gR_ & 31);
+#pragma unroll
+      for (int m = 0; m < K; ++m) out[m] = lds_tok(aR + 4 * m, tok);
+    }
+  };
+  bool rvn_valid = false;  // rvn must be (re)loaded after each chunk event (new token)
+#pragma unroll
+  for (int m = 0; m < K; ++m) negp[m] = static_cast<int>(opaque(static_cast<uint32_t>(negp[m])));
+
   // one wavefront step; ALL = every lane's row is in 1..n (steady state, no predicates)
   auto step = [&](const int sig, auto all_tag) {
     constexpr bool ALL = decltype(all_tag)::value;
@@ -333,9 +351,11 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
 #pragma unroll
       for (int m = 0; m < K; ++m) rv[m] = prmt_sext(pw, 0x8880u + 0x1111u * m);  // sign-extended byte m
     } else {
-      const uint32_t aR = laneR + roff + 4u * static_cast<uint32_t>(gR & 31);
+      if (!rvn_valid) load_ref(rvn, rr, gR);
 #pragma unroll
-      for (int m = 0; m < K; ++m) rv[m] = lds_tok(aR + 4 * m, tok);
+      for (int m = 0; m < K; ++m) rv[m] = rvn[m];
+      load_ref(rvn, rr + 1, gR + ldr32);  // next row (same chunk block or ring-resident)
+      rvn_valid = true;
     }
     const int bval = __shfl_sync(FULL, static_cast<int>(static_cast<uint32_t>(cur)), sig & 31);
     const int from_left = __shfl_up_sync(FULL, vlast, 1);
@@ -409,6 +429,7 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
       if (tracing) wait_cyc += clock64() - c_w0;
     }
     // event Q reached: score chunk Q-STORE_DELAY is complete, ref chunk Q-SKEW-1 no longer read
+    rvn_valid = false;  // rows of the new chunk may be read only after this event's wait
     __syncwarp();
     if (t == 0) mbar_arrive(bar_ev + 8 * (Q % C::SLOTS));
     if (sig0 >= nsteps) {
