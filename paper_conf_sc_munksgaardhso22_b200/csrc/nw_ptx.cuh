@@ -41,6 +41,9 @@ __device__ __forceinline__ void cp_async16_p(bool p, uint32_t dst, const void* s
                "r"(dst), "l"(src)
                : "memory");
 }
+__device__ __forceinline__ void prefetch_l2_p(bool p, const void* a) {
+  asm volatile("{ .reg .pred q; setp.ne.b32 q, %0, 0; @q prefetch.global.L2 [%1]; }" ::"r"(static_cast<int>(p)), "l"(a));
+}
 __device__ __forceinline__ int4 lds128_p(bool p, uint32_t a) {
   int4 v = make_int4(0, 0, 0, 0);
   asm volatile("{ .reg .pred q; setp.ne.b32 q, %4, 0; @q ld.shared.v4.b32 {%0, %1, %2, %3}, [%5]; }"

@@ -48,6 +48,7 @@ namespace nwb200 {
 constexpr int kBarBytes = 512;  // per band pair: ref_full[16], ev[16], st_done[16] mbarriers
 constexpr int kBR = 256;      // shared border ring entries between consecutive warps of a CTA
 constexpr int kRing = 64;     // rows per staging ring (power of two)
+constexpr int kPF = 4;        // ref chunks prefetched into L2 beyond the smem lookahead
 constexpr unsigned kErrWatchdog = 0xBADB0001u;
 
 // Geometry of one kernel instance.  Events happen every CH steps (event Q starts step CH*Q).
@@ -676,14 +677,22 @@ __device__ __forceinline__ void nw_stage(const StripParams& P, const long long t
     mbar_wait(bar_ev + 8 * sl, (ph_ev >> sl) & 1u);
     ph_ev ^= 1u << sl;
     wait_cyc += clock64() - c_w0;
+    if constexpr (!SEQ) {
+      if (Q + C::LOOKW < nch) issue_ref(Q + C::LOOKW);
+      // warm L2 with the ref rows kPF chunks further ahead: one 128-byte line per lane
+      const int cp = Q + C::LOOKW + kPF;
+      if (cp < nch) {
+        const int i = t / 4, ln = t % 4;  // CH = 8 rows x 4 lines (K=2: 2-3 lines per row)
+        const int r = cp * CH + 1 + i;
+        const uintptr_t g = reinterpret_cast<uintptr_t>(R + static_cast<long long>(r) * P.ldr + c0) + 128u * ln;
+        prefetch_l2_p(i < CH && r <= n && 128 * ln < 4 * ws + 128, reinterpret_cast<const void*>(g));
+      }
+    }
     const int cs = Q - C::STORE_DELAY;
     if (cs >= 0 && cs < nch) {
       store_sc(cs);
       __syncwarp();
       if (t == 0) mbar_arrive(bar_sd + 8 * (cs % C::SLOTS));
-    }
-    if constexpr (!SEQ) {
-      if (Q + C::LOOKW < nch) issue_ref(Q + C::LOOKW);
     }
   }
   if (P.trace2 != nullptr && t == 0 && task < P.trace_cap) {
