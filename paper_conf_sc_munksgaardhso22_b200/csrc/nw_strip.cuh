@@ -199,6 +199,7 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
   const long long c_task0 = clock64();
   const bool tracing = P.trace != nullptr;
   long long ev_cyc = 0, spin_cyc = 0, wait_cyc = 0;  // debug cycle accounting (trace only)
+  long long blk_cyc = 0;                              // steady-state step blocks
 
   const uint32_t s_prog = smem_u32(smem + 8);
   const uint32_t s_bring = smem_u32(smem + 128);
@@ -475,8 +476,10 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
     if (tracing) ev_cyc += clock64() - c_ev0;
     // ---- CH wavefront steps: lane t computes row sig+1-t, columns c0+tK .. c0+tK+K-1
     if (sig0 >= 31 && sig0 + CH <= n) {  // steady state: all 32 lanes on rows 1..n
+      const long long c_b0 = tracing ? clock64() : 0;
 #pragma unroll
       for (int j = 0; j < CH; ++j) step(sig0 + j, std::true_type{});
+      if (tracing) blk_cyc += clock64() - c_b0;
     } else {
 #pragma unroll 1
       for (int j = 0; j < CH; ++j) {
@@ -500,7 +503,7 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
     e[0] = static_cast<unsigned long long>(task);
     e[1] = t_task0;
     e[2] = globaltimer_ns();
-    e[3] = smid;
+    e[3] = (static_cast<unsigned long long>(blk_cyc) << 16) | smid;  // steady-block cycles << 16 | smid
     e[4] = static_cast<unsigned long long>(ev_cyc);    // cycles in chunk events (incl. waits)
     e[5] = static_cast<unsigned long long>(wait_cyc);  // of which: waits on the staging warp
     e[6] = static_cast<unsigned long long>(spin_cyc);  // of which: left-border spins

@@ -28,7 +28,11 @@ def main(path, n=None):
     grid = np.linspace(0, span, 21)
     act = [int(((st <= g) & (en > g)).sum()) for g in grid]
     print("bands in flight over the launch:", act)
+    blk = t[:, 3] >> 16
+    t[:, 3] &= 0xFFFF
     print("distinct SMs:", len(np.unique(t[:, 3])))
+    if n and blk.max() > 0:
+        print(f"  steady-state step blocks: mean {blk.mean() / n:.1f} cycles/row, band0 {blk[0] / n:.1f}")
     if t.shape[1] >= 8:
         tot = t[:, 7].astype(float)
         cols = [("events", 4), ("ref waits", 5), ("border spins", 6)]
