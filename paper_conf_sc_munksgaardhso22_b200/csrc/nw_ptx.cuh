@@ -75,6 +75,21 @@ __device__ __forceinline__ void stg128(void* p, int4 v) {
   asm volatile("st.global.v4.b32 [%0], {%1, %2, %3, %4};" ::"l"(p), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w) : "memory");
 }
 
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() {
+  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
+}
+// staging -> compute progress word {lo, hi} with release / acquire semantics at CTA scope
+__device__ __forceinline__ void st_release_cta_v2(uint32_t a, uint32_t lo, uint32_t hi) {
+  asm volatile("{ .reg .b64 e; mov.b64 e, {%1, %2}; st.release.cta.shared.b64 [%0], e; }" ::"r"(a), "r"(lo), "r"(hi) : "memory");
+}
+__device__ __forceinline__ uint64_t ld_acquire_cta(uint32_t a) {
+  uint64_t v;
+  asm volatile("ld.acquire.cta.shared.b64 %0, [%1];" : "=l"(v) : "r"(a) : "memory");
+  return v;
+}
+
 __device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
   asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count) : "memory");
 }

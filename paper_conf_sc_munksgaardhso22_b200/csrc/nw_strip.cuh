@@ -191,7 +191,7 @@ enum : int { kSinkNone = 0, kSinkSmem = 1, kSinkGlobal = 2 };
 template <class C, int SINK>
 __device__ __forceinline__ void nw_band(const StripParams& P, const long long task, const int w, const int t,
                                         unsigned char* const smem, unsigned char* const wsm, const uint32_t gen,
-                                        uint32_t& ph_rf, uint32_t& ph_sd) {
+                                        uint32_t& cbase) {
   constexpr int K = C::K, RS = C::RS, CH = C::CH;
   constexpr bool SEQ = C::SEQ;
   constexpr unsigned FULL = 0xffffffffu;
@@ -203,7 +203,7 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
 
   const uint32_t s_prog = smem_u32(smem + 8);
   const uint32_t s_bring = smem_u32(smem + 128);
-  const uint32_t bar_rf = smem_u32(wsm), bar_ev = bar_rf + 128, bar_sd = bar_rf + 256;
+  const uint32_t bar_ev = smem_u32(wsm) + 128, s_state = smem_u32(wsm) + 384;
   int32_t* const ref_ring = reinterpret_cast<int32_t*>(wsm + kBarBytes);
   int32_t* const sc_ring = ref_ring + C::REF_ROWS * RS;
   uint32_t* const prof = reinterpret_cast<uint32_t*>(sc_ring + kRing * RS);
@@ -285,9 +285,10 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
   for (int m = 0; m < K; ++m) Pv[m] = (t * K + m < ws) ? __ldg(S + c0 + t * K + m) : 0;
   int Lprev = (t * K < ws) ? __ldg(S + c0 + t * K - 1) : 0;  // diag input of the first row
   int vlast = Pv[K - 1];
-  int win_base = 1;  // cur holds border rows win_base + t
-  uint64_t cur = load_entry(1 + t);
-  uint64_t nxt = src == kSrcSmem ? 0ull : load_entry(33 + t);
+  // left border, per CH-row block: lane j < CH holds the entry of row sig0+1+j; the next
+  // block's entries are prefetched one block ahead (pend)
+  uint64_t cur = 0ull;
+  uint64_t pend = t < CH ? load_entry(1 + t) : 0ull;
   // per-lane ring addressing: row r (= step + 1 - t) lives at ring row (r-1) & 63
   const int r0 = 1 - t;
   int rr = r0 - 1;  // r - 1
@@ -359,7 +360,7 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
       load_ref(rvn, rr + 1, gR + ldr32);  // next row (same chunk block or ring-resident)
       rvn_valid = true;
     }
-    const int bval = __shfl_sync(FULL, static_cast<int>(static_cast<uint32_t>(cur)), sig & 31);
+    const int bval = __shfl_sync(FULL, static_cast<int>(static_cast<uint32_t>(cur)), sig & (CH - 1));
     const int from_left = __shfl_up_sync(FULL, vlast, 1);
     const int L = (t == 0) ? bval : from_left;
     bool active = true;
@@ -418,20 +419,30 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
     // ---- chunk events (warp-uniform).  The paired staging warp stores finished score chunks
     // and prefetches ref chunks; this warp only synchronises with it.
     if (Q < nch) {
+      // staging progress: ref chunk Q in shared memory, score chunk Q-SLOTS stored (its slot
+      // is about to be rewritten)
       const long long c_w0 = tracing ? clock64() : 0;
-      const int sl = Q % C::SLOTS;
-      if (Q >= C::SLOTS) {  // score slot of chunk Q is free once chunk Q-SLOTS was stored
-        mbar_wait(bar_sd + 8 * sl, (ph_sd >> sl) & 1u);
-        ph_sd ^= 1u << sl;
+      const uint32_t need_rd = cbase + static_cast<uint32_t>(Q) + 1u;
+      const uint32_t need_st = Q >= C::SLOTS ? cbase + static_cast<uint32_t>(Q - C::SLOTS) + 1u : 0u;
+      uint64_t stt = ld_acquire_cta(s_state);
+      auto ok = [&](uint64_t v) {
+        return (SEQ || static_cast<int>(static_cast<uint32_t>(v) - need_rd) >= 0) &&
+               static_cast<int>(static_cast<uint32_t>(v >> 32) - need_st) >= 0;
+      };
+      if (!ok(stt)) {
+        const uint64_t t0 = globaltimer_ns();
+        unsigned spins = 0;
+        do {
+          stt = ld_acquire_cta(s_state);
+          if ((++spins & 1023u) == 0 && globaltimer_ns() - t0 > P.spin_limit_ns) watchdog_trap(P.err);
+        } while (!ok(stt));
       }
-      if constexpr (!SEQ) {
-        tok = mbar_wait_tok(bar_rf + 8 * sl, (ph_rf >> sl) & 1u);
-        ph_rf ^= 1u << sl;
-      }
+      // token (always 0) data-dependent on the acquire: the ref loads cannot move above it
+      asm volatile("and.b32 %0, %1, 0;" : "=r"(tok) : "r"(static_cast<uint32_t>(stt)));
       if (tracing) wait_cyc += clock64() - c_w0;
     }
     // event Q reached: score chunk Q-STORE_DELAY is complete, ref chunk Q-SKEW-1 no longer read
-    rvn_valid = false;  // rows of the new chunk may be read only after this event's wait
+    rvn_valid = false;  // rows of the new chunk may be read only after this event's check
     __syncwarp();
     if (t == 0) mbar_arrive(bar_ev + 8 * (Q % C::SLOTS));
     if (sig0 >= nsteps) {
@@ -439,17 +450,13 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
       continue;
     }
     if (src == kSrcSmem && t == 0) sts32_volatile(prog_in, sig0);  // rows <= sig0 consumed
-    if ((sig0 & 31) == 0 && sig0 > 0) {
-      cur = src == kSrcSmem ? load_entry(sig0 + 1 + t) : nxt;
-      win_base = sig0 + 1;
-      if (src != kSrcSmem) nxt = load_entry(sig0 + 33 + t);
-    }
+    cur = pend;
+    pend = (t < CH) ? load_entry(sig0 + CH + 1 + t) : 0ull;  // next block, one block ahead
     if (src != kSrcPlain) {
-      // the block needs rows sig0+1 .. sig0+CH of the left border (lanes j0 .. j0+CH-1)
-      const int j0 = sig0 & 31;
+      // the block needs rows sig0+1 .. sig0+CH of the left border (lanes 0 .. CH-1)
       auto ready = [&]() {
-        const int row = win_base + t;
-        const bool need = t >= j0 && t < j0 + CH && row <= n;
+        const int row = sig0 + 1 + t;
+        const bool need = t < CH && row <= n;
         return __all_sync(FULL, !need || entry_ok(cur, row)) != 0;
       };
       if (!ready()) {
@@ -457,7 +464,7 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
         const uint64_t t0 = globaltimer_ns();
         unsigned spins = 0;
         do {
-          cur = load_entry(win_base + t);
+          cur = t < CH ? load_entry(sig0 + 1 + t) : 0ull;
           if ((++spins & 255u) == 0 && globaltimer_ns() - t0 > P.spin_limit_ns) watchdog_trap(P.err);
         } while (!ready());
         spin_cyc += clock64() - c_0;
@@ -488,13 +495,7 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
       }
     }
   }
-  // consume the staging warp's remaining "stored" arrivals (chunks nch-SLOTS .. nch-1) so the
-  // st_done phases stay in step across tasks
-  for (int c = max(0, nch - C::SLOTS); c < nch; ++c) {
-    const int sl = c % C::SLOTS;
-    mbar_wait(bar_sd + 8 * sl, (ph_sd >> sl) & 1u);
-    ph_sd ^= 1u << sl;
-  }
+  cbase += static_cast<uint32_t>(nch);
   __syncwarp();
   if (P.trace != nullptr && t == 0 && task < P.trace_cap) {
     unsigned smid;
@@ -516,12 +517,12 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
 // finished score chunks, driven by the compute warp's per-event mbarrier arrivals.
 template <class C>
 __device__ __forceinline__ void nw_stage(const StripParams& P, const long long task, const int t,
-                                         unsigned char* const wsm, uint32_t& ph_ev) {
+                                         unsigned char* const wsm, uint32_t& ph_ev, uint32_t& cbase) {
   constexpr int RS = C::RS, CH = C::CH;
   constexpr bool SEQ = C::SEQ;
   const long long c_task0 = clock64();
   long long wait_cyc = 0;
-  const uint32_t bar_rf = smem_u32(wsm), bar_ev = bar_rf + 128, bar_sd = bar_rf + 256;
+  const uint32_t bar_ev = smem_u32(wsm) + 128, s_state = smem_u32(wsm) + 384;
   int32_t* const ref_ring = reinterpret_cast<int32_t*>(wsm + kBarBytes);
   int32_t* const sc_ring = ref_ring + C::REF_ROWS * RS;
   const int n = static_cast<int>(P.n);
@@ -539,7 +540,6 @@ __device__ __forceinline__ void nw_stage(const StripParams& P, const long long t
       SEQ ? 0 : reinterpret_cast<uintptr_t>(R + static_cast<long long>(n) * P.ldr + P.width + 1);  // past the last element
   const uint32_t refR0 = opaque(smem_u32(ref_ring));
   const uint32_t scR0 = opaque(smem_u32(sc_ring));
-  const uint32_t bar0 = bar_rf;
 
   // Per-lane staging assignments, fixed for the whole task: in iteration it lane t moves the
   // 16-byte chunk k of row i of a CH-row chunk (f = t + 32*it, i = f / MAX, k = f % MAX).  Chunk c
@@ -597,7 +597,6 @@ __device__ __forceinline__ void nw_stage(const StripParams& P, const long long t
         }
       }
     }
-    cp_async_arrive(bar0 + 8 * (c % C::SLOTS));
   };
 
   // score stores, same scheme: interior 16-byte chunks (all LDS.128 first, then STG.128) and
@@ -671,9 +670,19 @@ __device__ __forceinline__ void nw_stage(const StripParams& P, const long long t
     }
   };
 
+  // progress published to the compute warp: ref chunks < rd are in shared memory, score
+  // chunks < sd are stored (absolute chunk numbers, cbase = chunks of earlier tasks)
+  uint32_t rd = cbase, sd = cbase;
   if constexpr (!SEQ) {
-    for (int c = 0; c < C::LOOKW && c < nch; ++c) issue_ref(c);
+    for (int c = 0; c < C::LOOKW; ++c) {
+      if (c < nch) issue_ref(c);
+      cp_async_commit();  // one group per chunk (possibly empty)
+    }
+    cp_async_wait<C::LOOKW - 1>();  // chunk 0 landed
+    rd = cbase + 1;
   }
+  __syncwarp();
+  if (t == 0) st_release_cta_v2(s_state, rd, sd);
   for (int Q = 0; Q <= nch + C::STORE_DELAY - 1; ++Q) {
     const int sl = Q % C::SLOTS;
     const long long c_w0 = clock64();
@@ -682,10 +691,11 @@ __device__ __forceinline__ void nw_stage(const StripParams& P, const long long t
     wait_cyc += clock64() - c_w0;
     if constexpr (!SEQ) {
       if (Q + C::LOOKW < nch) issue_ref(Q + C::LOOKW);
+      cp_async_commit();
       // warm L2 with the ref rows kPF chunks further ahead: one 128-byte line per lane
       const int cp = Q + C::LOOKW + kPF;
       if (cp < nch) {
-        const int i = t / 4, ln = t % 4;  // CH = 8 rows x 4 lines (K=2: 2-3 lines per row)
+        const int i = t / 4, ln = t % 4;
         const int r = cp * CH + 1 + i;
         const uintptr_t g = reinterpret_cast<uintptr_t>(R + static_cast<long long>(r) * P.ldr + c0) + 128u * ln;
         prefetch_l2_p(i < CH && r <= n && 128 * ln < 4 * ws + 128, reinterpret_cast<const void*>(g));
@@ -694,10 +704,16 @@ __device__ __forceinline__ void nw_stage(const StripParams& P, const long long t
     const int cs = Q - C::STORE_DELAY;
     if (cs >= 0 && cs < nch) {
       store_sc(cs);
-      __syncwarp();
-      if (t == 0) mbar_arrive(bar_sd + 8 * (cs % C::SLOTS));
+      sd = cbase + static_cast<uint32_t>(cs) + 1u;
     }
+    if constexpr (!SEQ) {
+      cp_async_wait<C::LOOKW - 1>();  // chunks <= Q+1 landed
+      rd = cbase + static_cast<uint32_t>(min(Q + 2, nch));
+    }
+    __syncwarp();  // every lane's copies / stores of this iteration are done
+    if (t == 0) st_release_cta_v2(s_state, rd, sd);
   }
+  cbase += static_cast<uint32_t>(nch);
   if (P.trace2 != nullptr && t == 0 && task < P.trace_cap) {
     P.trace2[2 * task] = static_cast<unsigned long long>(clock64() - c_task0);
     P.trace2[2 * task + 1] = static_cast<unsigned long long>(wait_cyc);
@@ -718,11 +734,8 @@ __global__ void __launch_bounds__(64 * C::NW, 1) nw_strip_kernel(const __grid_co
   unsigned char* const wsm = smem + C::kCtaHdr + w * C::kWarpSmem;
   if (!staging && t == 0) {
     const uint32_t b = smem_u32(wsm);
-    for (int i = 0; i < C::SLOTS; ++i) {
-      mbar_init(b + 8 * i, 32);        // ref_full: one cp.async arrival per staging lane
-      mbar_init(b + 128 + 8 * i, 1);   // ev: the compute warp reached an event
-      mbar_init(b + 256 + 8 * i, 1);   // st_done: the staging warp stored a score chunk
-    }
+    for (int i = 0; i < C::SLOTS; ++i) mbar_init(b + 128 + 8 * i, 1);  // ev: the compute warp reached an event
+    st_release_cta_v2(b + 384, 0u, 0u);                                 // staging progress word
   }
   fence_mbar_init();
   // shared border rings start invalid (tag 0xFFFFFFFF never equals gen | row, row < 2^30)
@@ -730,7 +743,8 @@ __global__ void __launch_bounds__(64 * C::NW, 1) nw_strip_kernel(const __grid_co
   if (threadIdx.x < NW) sts32_volatile(s_prog + 4 * threadIdx.x, 0);
   __syncthreads();
 
-  uint32_t ph_a = 0, ph_b = 0;  // mbarrier phase bits this warp waits on
+  uint32_t ph_a = 0;   // mbarrier phase bits this warp waits on (staging: ev)
+  uint32_t cbase = 0;  // chunks of earlier tasks (absolute chunk numbering shared by a warp pair)
   int gcount = 0;               // groups processed by this CTA (generation of the shared border tags)
   for (;;) {
     if (threadIdx.x == 0) *s_group = atomicAdd(P.ticket, 1ull);
@@ -741,7 +755,7 @@ __global__ void __launch_bounds__(64 * C::NW, 1) nw_strip_kernel(const __grid_co
     const uint32_t gen = static_cast<uint32_t>(gcount & 3) << 30;
     if (task < P.ntasks) {
       if (staging) {
-        nw_stage<C>(P, task, t, wsm, ph_a);
+        nw_stage<C>(P, task, t, wsm, ph_a, cbase);
       } else {
         const int band = static_cast<int>(task % P.nbands);
         const bool last_band = band == P.nbands - 1;
@@ -751,11 +765,11 @@ __global__ void __launch_bounds__(64 * C::NW, 1) nw_strip_kernel(const __grid_co
         else
           sink = (w < NW - 1) ? kSinkSmem : kSinkGlobal;
         if (sink == kSinkSmem)
-          nw_band<C, kSinkSmem>(P, task, w, t, smem, wsm, gen, ph_a, ph_b);
+          nw_band<C, kSinkSmem>(P, task, w, t, smem, wsm, gen, cbase);
         else if (sink == kSinkGlobal)
-          nw_band<C, kSinkGlobal>(P, task, w, t, smem, wsm, gen, ph_a, ph_b);
+          nw_band<C, kSinkGlobal>(P, task, w, t, smem, wsm, gen, cbase);
         else
-          nw_band<C, kSinkNone>(P, task, w, t, smem, wsm, gen, ph_a, ph_b);
+          nw_band<C, kSinkNone>(P, task, w, t, smem, wsm, gen, cbase);
       }
     }
     __syncthreads();  // group end: every warp done (shared border rings / progress reusable)
