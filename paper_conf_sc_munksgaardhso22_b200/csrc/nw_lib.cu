@@ -208,6 +208,13 @@ nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* 
   P.ticket = w->d_ticket;
   P.err = w->d_err;
   P.spin_limit_ns = spin_limit_ns();
+  {
+    static const unsigned dbg = [] {
+      const char* e = std::getenv("NW_DEBUG_SKIP");
+      return e ? static_cast<unsigned>(std::strtoul(e, nullptr, 0)) : 0u;
+    }();
+    P.dbg_skip = dbg;
+  }
   P.trace = g_trace;
   P.trace_cap = g_trace_cap;
   P.trace2 = g_trace ? g_trace + 8 * g_trace_cap : nullptr;

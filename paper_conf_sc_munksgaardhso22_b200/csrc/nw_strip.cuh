@@ -114,6 +114,7 @@ struct StripParams {
   unsigned long long* trace;  // debug: per task 8 x u64 (see nw.h nw_debug_set_trace) or null
   long long trace_cap;
   unsigned long long* trace2;  // debug: per task {store cycles, ref-issue cycles} or null
+  unsigned int dbg_skip;       // timing experiments only (results invalid when nonzero)
   // NEXT-2 (SEQ kernels): ref[i][j] = subst[a[i-1]][b[j-1]] generated on chip
   const uint8_t* seq_a;
   const uint8_t* seq_b;
@@ -418,7 +419,7 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
     const long long c_ev0 = tracing ? clock64() : 0;
     // ---- chunk events (warp-uniform).  The paired staging warp stores finished score chunks
     // and prefetches ref chunks; this warp only synchronises with it.
-    if (Q < nch) {
+    if (Q < nch && !(P.dbg_skip & 2u)) {
       // staging progress: ref chunk Q in shared memory, score chunk Q-SLOTS stored (its slot
       // is about to be rewritten)
       const long long c_w0 = tracing ? clock64() : 0;
@@ -444,7 +445,7 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
     // event Q reached: score chunk Q-STORE_DELAY is complete, ref chunk Q-SKEW-1 no longer read
     rvn_valid = false;  // rows of the new chunk may be read only after this event's check
     __syncwarp();
-    if (t == 0) mbar_arrive(bar_ev + 8 * (Q % C::SLOTS));
+    if (t == 0 && !(P.dbg_skip & 4u)) mbar_arrive(bar_ev + 8 * (Q % C::SLOTS));
     if (sig0 >= nsteps) {
       if (tracing) ev_cyc += clock64() - c_ev0;
       continue;
@@ -452,7 +453,7 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
     if (src == kSrcSmem && t == 0) sts32_volatile(prog_in, sig0);  // rows <= sig0 consumed
     cur = pend;
     pend = (t < CH) ? load_entry(sig0 + CH + 1 + t) : 0ull;  // next block, one block ahead
-    if (src != kSrcPlain) {
+    if (src != kSrcPlain && !(P.dbg_skip & 8u)) {
       // the block needs rows sig0+1 .. sig0+CH of the left border (lanes 0 .. CH-1)
       auto ready = [&]() {
         const int row = sig0 + 1 + t;
@@ -670,6 +671,10 @@ __device__ __forceinline__ void nw_stage(const StripParams& P, const long long t
     }
   };
 
+  if (P.dbg_skip & 1u) {
+    cbase += static_cast<uint32_t>(nch);
+    return;
+  }
   // progress published to the compute warp: ref chunks < rd are in shared memory, score
   // chunks < sd are stored (absolute chunk numbers, cbase = chunks of earlier tasks)
   uint32_t rd = cbase, sd = cbase;
