@@ -286,10 +286,12 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
   for (int m = 0; m < K; ++m) Pv[m] = (t * K + m < ws) ? __ldg(S + c0 + t * K + m) : 0;
   int Lprev = (t * K < ws) ? __ldg(S + c0 + t * K - 1) : 0;  // diag input of the first row
   int vlast = Pv[K - 1];
-  // left border, per CH-row block: lane j < CH holds the entry of row sig0+1+j; the next
-  // block's entries are prefetched one block ahead (pend)
+  // left border, per CH-row block: lane j < CH holds the entry of row sig0+1+j.  Entries are
+  // prefetched D blocks ahead (lanes CH*d .. CH*d+CH-1 of `pend` hold block Q+d, d < D): deep
+  // for the read-only plain column, shallow for handoffs that are published just in time.
+  const int D = src == kSrcPlain ? 3 : (src == kSrcGlobal ? 2 : 1);
   uint64_t cur = 0ull;
-  uint64_t pend = t < CH ? load_entry(1 + t) : 0ull;
+  uint64_t pend = t < CH * D ? load_entry(1 + t) : 0ull;  // blocks 0 .. D-1
   // per-lane ring addressing: row r (= step + 1 - t) lives at ring row (r-1) & 63
   const int r0 = 1 - t;
   int rr = r0 - 1;  // r - 1
@@ -451,8 +453,14 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
       continue;
     }
     if (src == kSrcSmem && t == 0) sts32_volatile(prog_in, sig0);  // rows <= sig0 consumed
+    // rotate the prefetch window down by one block (lanes CH.. -> 0..), load block Q+D on top
     cur = pend;
-    pend = (t < CH) ? load_entry(sig0 + CH + 1 + t) : 0ull;  // next block, one block ahead
+    {
+      const uint32_t lo = __shfl_down_sync(FULL, static_cast<uint32_t>(pend), CH);
+      const uint32_t hi = __shfl_down_sync(FULL, static_cast<uint32_t>(pend >> 32), CH);
+      pend = (static_cast<uint64_t>(hi) << 32) | lo;
+      if (t >= CH * (D - 1) && t < CH * D) pend = load_entry(sig0 + CH * D + 1 + (t - CH * (D - 1)));
+    }
     if (src != kSrcPlain && !(P.dbg_skip & 8u)) {
       // the block needs rows sig0+1 .. sig0+CH of the left border (lanes 0 .. CH-1)
       auto ready = [&]() {
