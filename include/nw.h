@@ -96,8 +96,9 @@ nw_status nw_fill_batch_ld(int32_t* score, int64_t ld_score, int64_t stride_scor
  *   local score row 0 = global row 0 columns col0..col0+w (col 0 = the corner (0, col0));
  *   local score column 0, rows >= 1: the global left border (read only when halo_in == NULL,
  *   i.e. on rank 0); local ref column 0 unused.
- * halo_in  : (n+1) uint64 entries on THIS device, written by rank g-1's kernel
- *            (entry i = (epoch << 32) | (uint32) score[i][col0]); NULL on rank 0.
+ * halo_in  : n+2 uint64 entries on THIS device, 16-byte aligned, written by rank g-1's
+ *            kernel (entry i = (epoch << 32) | (uint32) score[i][col0], i = 1..n; the kernel
+ *            reads entries in 16-byte pairs, hence the spare entry n+1); NULL on rank 0.
  *            Must be zero-filled once before first use; never needs resetting after.
  * halo_out : rank g+1's halo_in (a peer-mapped pointer, e.g. torch symmetric memory) or
  *            NULL on the last rank.  A rank with halo_out needs w % nw_band_width(tile) == 0

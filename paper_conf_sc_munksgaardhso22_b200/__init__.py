@@ -166,7 +166,7 @@ def nw_fill_sharded(score, ref, penalty: int, *, halo_in=None, halo_out=None, ep
                     halo_out_is_peer: bool = False, tile: int = 0, stream=None):
     """One rank's column strip.  score/ref: local (n+1, >= w+1) int32 CUDA tensors.
 
-    halo_in: None (rank 0: left border = score[:, 0]) or an int64 CUDA tensor of n+1 tagged
+    halo_in: None (rank 0: left border = score[:, 0]) or an int64 CUDA tensor of n+2 tagged
     entries written by the left neighbour.  halo_out: None, an int64 tensor (same device) or an
     integer device address (peer-mapped, e.g. from torch symmetric memory)."""
     import torch
@@ -180,8 +180,8 @@ def nw_fill_sharded(score, ref, penalty: int, *, halo_in=None, halo_out=None, ep
             return None
         if isinstance(h, int):
             return h
-        if h.dtype not in (torch.int64, torch.uint64) or not h.is_cuda or h.numel() < n + 1:
-            raise ValueError("halo tensors must be int64 CUDA tensors with >= n+1 entries")
+        if h.dtype not in (torch.int64, torch.uint64) or not h.is_cuda or h.numel() < n + 2:
+            raise ValueError("halo tensors must be int64 CUDA tensors with >= n+2 entries")
         return h.data_ptr()
 
     st = NwStrip(score.data_ptr(), score.stride(0), ref.data_ptr(), ref.stride(0), n, w,

@@ -182,7 +182,8 @@ nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* 
   s = get_ws(dev, st, &w);
   if (s != NW_OK) return s;
   const int64_t nbands = (width + W - 1) / W;
-  const size_t entries = static_cast<size_t>(pairs) * static_cast<size_t>(nbands - 1) * static_cast<size_t>(n + 1);
+  // +2: the kernel's 16-byte border prefetches read entry pairs (2k, 2k+1), up to row n+1
+  const size_t entries = static_cast<size_t>(pairs) * static_cast<size_t>(nbands - 1) * static_cast<size_t>(n + 1) + 2;
   s = ensure_xbuf(w, entries, st);
   if (s != NW_OK) return s;
   StripParams P{};
@@ -371,7 +372,7 @@ nw_status nw_fill_sharded(const nw_strip* sp, int32_t penalty, int32_t tile, voi
   if (!aligned4(S.score) || !aligned4(S.ref)) return NW_EINVAL;
   if (overlaps(S.score, 4 * (S.n * S.ld_score + S.w + 1), S.ref, 4 * (S.n * S.ld_ref + S.w + 1))) return NW_EINVAL;
   if ((S.halo_in || S.halo_out) && S.epoch == 0) return NW_ECOMM;
-  if ((S.halo_in && (reinterpret_cast<uintptr_t>(S.halo_in) & 7)) ||
+  if ((S.halo_in && (reinterpret_cast<uintptr_t>(S.halo_in) & 15)) ||
       (S.halo_out && (reinterpret_cast<uintptr_t>(S.halo_out) & 7)))
     return NW_ECOMM;
   // a strip that pushes a halo must end on a band boundary (its last band is then full width)

@@ -27,6 +27,16 @@ __device__ __forceinline__ void sts_s32(uint32_t a, int v) {
 __device__ __forceinline__ void cp_async16(uint32_t dst, const void* src) {
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst), "l"(src) : "memory");
 }
+__device__ __forceinline__ void cp_async16_cg_p(bool p, uint32_t dst, const void* src) {
+  asm volatile("{ .reg .pred q; setp.ne.b32 q, %0, 0; @q cp.async.cg.shared.global [%1], [%2], 16; }" ::"r"(static_cast<int>(p)),
+               "r"(dst), "l"(src)
+               : "memory");
+}
+__device__ __forceinline__ void cp_async4_p(bool p, uint32_t dst, const void* src) {
+  asm volatile("{ .reg .pred q; setp.ne.b32 q, %0, 0; @q cp.async.ca.shared.global [%1], [%2], 4; }" ::"r"(static_cast<int>(p)),
+               "r"(dst), "l"(src)
+               : "memory");
+}
 __device__ __forceinline__ void cp_async4(uint32_t dst, const void* src) {
   asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(dst), "l"(src) : "memory");
 }

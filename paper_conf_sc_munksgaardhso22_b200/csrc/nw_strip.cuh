@@ -45,7 +45,7 @@
 
 namespace nwb200 {
 
-constexpr int kBarBytes = 512;  // per band pair: ref_full[16], ev[16], st_done[16] mbarriers
+constexpr int kBarBytes = 1024;  // per band pair: ev mbarriers [128,256), progress word [384], border prefetch ring [512,1024)
 constexpr int kBR = 256;      // shared border ring entries between consecutive warps of a CTA
 constexpr int kRing = 64;     // rows per staging ring (power of two)
 constexpr int kPF = 4;        // ref chunks prefetched into L2 beyond the smem lookahead
@@ -286,12 +286,28 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
   for (int m = 0; m < K; ++m) Pv[m] = (t * K + m < ws) ? __ldg(S + c0 + t * K + m) : 0;
   int Lprev = (t * K < ws) ? __ldg(S + c0 + t * K - 1) : 0;  // diag input of the first row
   int vlast = Pv[K - 1];
-  // left border, per CH-row block: lane j < CH holds the entry of row sig0+1+j.  Entries are
-  // prefetched D blocks ahead (lanes CH*d .. CH*d+CH-1 of `pend` hold block Q+d, d < D): deep
-  // for the read-only plain column, shallow for handoffs that are published just in time.
-  const int D = src == kSrcPlain ? 3 : (src == kSrcGlobal ? 2 : 1);
+  // left border, per CH-row block: lane j < CH holds the entry of row sig0+1+j (`cur`).
+  // Global / plain sources are prefetched D blocks ahead by cp.async into a 4-block shared ring
+  // (no register scoreboard on the in-flight loads); a shared-ring source (warp w-1) is read
+  // directly at the event.  Ring slot of block q: entries of rows CH*q .. CH*q+CH+1.
+  constexpr int D = 2;
+  constexpr uint32_t kSlotB = 8u * (CH + 2);
+  const uint32_t bpre = smem_u32(wsm) + 512;
+  auto prefetch_block = [&](int q) {  // block q = rows CH*q+1 .. CH*q+CH
+    const uint32_t slot = bpre + kSlotB * static_cast<uint32_t>(q & 3);
+    if (src == kSrcGlobal) {
+      // 16-byte pairs (rows 2k, 2k+1) through L2 only (entries are polled: never via L1)
+      const int row = CH * q + 2 * t;
+      cp_async16_cg_p(t <= CH / 2 && row <= n, slot + 16u * t, lin + row);
+    } else if (src == kSrcPlain) {
+      const int row = CH * q + 1 + t;
+      cp_async4_p(t < CH && row <= n, slot + 8u * (1 + t), colp + static_cast<long long>(row) * P.lds);
+    }
+    cp_async_commit();
+  };
   uint64_t cur = 0ull;
-  uint64_t pend = t < CH * D ? load_entry(1 + t) : 0ull;  // blocks 0 .. D-1
+  if (src != kSrcSmem)
+    for (int q = 0; q < D; ++q) prefetch_block(q);
   // per-lane ring addressing: row r (= step + 1 - t) lives at ring row (r-1) & 63
   const int r0 = 1 - t;
   int rr = r0 - 1;  // r - 1
@@ -363,7 +379,7 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
       load_ref(rvn, rr + 1, gR + ldr32);  // next row (same chunk block or ring-resident)
       rvn_valid = true;
     }
-    const int bval = __shfl_sync(FULL, static_cast<int>(static_cast<uint32_t>(cur)), sig & (CH - 1));
+    const int bval = __shfl_sync(FULL, static_cast<int>(static_cast<uint32_t>(cur)), sig & (CH - 1));  // lane 0's left
     const int from_left = __shfl_up_sync(FULL, vlast, 1);
     const int L = (t == 0) ? bval : from_left;
     bool active = true;
@@ -453,13 +469,14 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
       continue;
     }
     if (src == kSrcSmem && t == 0) sts32_volatile(prog_in, sig0);  // rows <= sig0 consumed
-    // rotate the prefetch window down by one block (lanes CH.. -> 0..), load block Q+D on top
-    cur = pend;
-    {
-      const uint32_t lo = __shfl_down_sync(FULL, static_cast<uint32_t>(pend), CH);
-      const uint32_t hi = __shfl_down_sync(FULL, static_cast<uint32_t>(pend >> 32), CH);
-      pend = (static_cast<uint64_t>(hi) << 32) | lo;
-      if (t >= CH * (D - 1) && t < CH * D) pend = load_entry(sig0 + CH * D + 1 + (t - CH * (D - 1)));
+    if (src == kSrcSmem) {
+      cur = t < CH ? lds64_volatile(bring_in + 8u * ((sig0 + 1 + t) & (kBR - 1))) : 0ull;
+    } else {
+      cp_async_wait<D - 1>();  // block Q's entries landed (one group per block, D in flight)
+      __syncwarp();
+      cur = t < CH ? lds64_volatile(bpre + kSlotB * static_cast<uint32_t>(Q & 3) + 8u * (1 + t)) : 0ull;
+      __syncwarp();
+      prefetch_block(Q + D);  // into the slot of block Q+D-4, consumed two events ago
     }
     if (src != kSrcPlain && !(P.dbg_skip & 8u)) {
       // the block needs rows sig0+1 .. sig0+CH of the left border (lanes 0 .. CH-1)
@@ -473,7 +490,7 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
         const uint64_t t0 = globaltimer_ns();
         unsigned spins = 0;
         do {
-          cur = t < CH ? load_entry(sig0 + 1 + t) : 0ull;
+          cur = t < CH ? load_entry(sig0 + 1 + t) : 0ull;  // synchronous re-poll
           if ((++spins & 255u) == 0 && globaltimer_ns() - t0 > P.spin_limit_ns) watchdog_trap(P.err);
         } while (!ready());
         spin_cyc += clock64() - c_0;

@@ -107,7 +107,7 @@ class StripShard:
         self.device = torch.device("cuda", torch.cuda.current_device())
         self.strip = strip_bounds(n, self.world)[self.rank]
         self.score, self.ref = local_strip_problem(n, p, seed, self.strip, self.device)
-        self.halo = symm_mem.empty(n + 1, dtype=torch.int64, device=self.device)
+        self.halo = symm_mem.empty(n + 2, dtype=torch.int64, device=self.device)  # n+2 entries (nw.h)
         self.halo.zero_()
         torch.cuda.synchronize()
         self.hdl = symm_mem.rendezvous(self.halo, self.group)

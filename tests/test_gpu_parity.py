@@ -157,7 +157,7 @@ def test_sharded_single_device(G, n, tile):
     score, ref = inputs.make_problem(n, 10, seed=17)
     want = expect(score, ref, 10)
     strips = split_strips(score, ref, G, tile)
-    halos = [torch.zeros(n + 1, dtype=torch.int64, device="cuda") for _ in range(G + 1)]
+    halos = [torch.zeros(n + 2, dtype=torch.int64, device="cuda") for _ in range(G + 1)]  # n+2: see nw.h
     for epoch in (1, 2, 7):                        # re-use of halo buffers across calls
         locs = []
         for g, (a, b, ls, lr) in enumerate(strips):
