@@ -183,7 +183,7 @@ nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* 
   if (s != NW_OK) return s;
   const int64_t nbands = (width + W - 1) / W;
   // +2: the kernel's 16-byte border prefetches read entry pairs (2k, 2k+1), up to row n+1
-  const size_t entries = static_cast<size_t>(pairs) * static_cast<size_t>(nbands - 1) * static_cast<size_t>(n + 1) + 2;
+  const size_t entries = static_cast<size_t>(pairs) * static_cast<size_t>(nbands - 1) * static_cast<size_t>(xstride(n)) + 2;
   s = ensure_xbuf(w, entries, st);
   if (s != NW_OK) return s;
   StripParams P{};

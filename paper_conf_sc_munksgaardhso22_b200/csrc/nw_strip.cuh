@@ -89,6 +89,9 @@ __host__ __device__ __forceinline__ int band_ws(long long width, int band, int W
   return static_cast<int>(r < W ? r : W);
 }
 __host__ __device__ __forceinline__ int lane_row(int step, int lane) { return step + 1 - lane; }
+// entries per band-border slot in the global border buffer: >= n+2 (16-byte pair reads may touch
+// row n+1) and even (every slot starts 16-byte aligned)
+__host__ __device__ __forceinline__ long long xstride(long long n) { return (n + 3) & ~1ll; }
 
 struct StripParams {
   int32_t* score;
@@ -235,7 +238,7 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
     src = kSrcSmem;  // band-1 is warp w-1 of this CTA
   } else {
     src = kSrcGlobal;
-    lin = P.xbuf + (pair * (P.nbands - 1) + band - 1) * static_cast<long long>(n + 1);
+    lin = P.xbuf + (pair * (P.nbands - 1) + band - 1) * xstride(n);
     lin_epoch = P.epoch;
   }
   // ---- sink (right)
@@ -248,7 +251,7 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
       lout_tag = P.halo_epoch;
       lout_sys = P.halo_out_sys != 0;
     } else {
-      lout = P.xbuf + (pair * (P.nbands - 1) + band) * static_cast<long long>(n + 1);
+      lout = P.xbuf + (pair * (P.nbands - 1) + band) * xstride(n);
       lout_tag = P.epoch;
     }
   } else if constexpr (SINK == kSinkSmem) {
