@@ -42,5 +42,30 @@ def main():
     print(json.dumps(res))
 
 
-if __name__ == "__main__":
+if __name__ == "__main__" and not (len(sys.argv) > 3 and sys.argv[3] == "global"):
     main()
+
+
+def global_source_probe(n=32768, tile=128, epoch=5):
+    """One band whose left border comes from an already-published (valid) global halo."""
+    W = nwb.nw_band_width(tile)
+    S, R = inputs.device_problem(n, 10, device="cuda")
+    S1, R1 = S[:, : W + 1], R[:, : W + 1]
+    vals = S[:, 0].to(torch.int64) & 0xFFFFFFFF
+    halo = torch.zeros(n + 2, dtype=torch.int64, device="cuda")
+    halo[: n + 1] = (epoch << 32) | vals
+    for label, kw in (("plain", {}), ("global halo", {"halo_in": halo, "epoch": epoch})):
+        for _ in range(2):
+            nwb.nw_fill_sharded(S1, R1, 10, tile=tile, **kw)
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        for _ in range(3):
+            nwb.nw_fill_sharded(S1, R1, 10, tile=tile, **kw)
+        e1.record()
+        torch.cuda.synchronize()
+        print(f"1 band, {label:12s}: {e0.elapsed_time(e1) / 3:.3f} ms", flush=True)
+
+
+if __name__ == "__main__" and len(sys.argv) > 3 and sys.argv[3] == "global":
+    global_source_probe(int(sys.argv[1]), int(sys.argv[2]))

@@ -175,7 +175,7 @@ def test_sharded_single_device(G, n, tile):
             got = locs[g].cpu().numpy()
             np.testing.assert_array_equal(got[:, 1:], want[:, a + 1:b + 1], err_msg=f"strip {g} epoch {epoch}")
         # halo entries carry the tag and the left neighbour's last column
-        h = halos[1].cpu().numpy().view(np.uint64)
+        h = halos[1].cpu().numpy().view(np.uint64)[: n + 1]
         assert (h[1:] >> np.uint64(32) == epoch).all()
         np.testing.assert_array_equal((h[1:] & np.uint64(0xFFFFFFFF)).astype(np.uint32).view(np.int32),
                                       want[1:, strips[0][1]])
