@@ -188,8 +188,9 @@ void nw_debug_set_grid(int32_t grid);
 
 /* Debug hook: persistent-kernel launches record, per task (pair, band) t < cap_tasks, eight
  * uint64 {t, start_ns, end_ns, smid, event_cycles, ref_wait_cycles, border_spin_cycles,
- * total_cycles} into the DEVICE buffer dev_buf (NULL = off); dev_buf must hold 10 * cap_tasks
- * uint64 (the tail gets {store_cycles, ref_issue_cycles} per task).
+ * total_cycles} into the DEVICE buffer dev_buf (NULL = off); dev_buf must hold 16 * cap_tasks
+ * uint64 (the tail gets 8 more counters per task: staging busy / wait cycles and the compute
+ * warp's event sub-phases).
  * Used by bench.py --trace to measure the wavefront ramp and the band-to-band lag. */
 void nw_debug_set_trace(uint64_t* dev_buf, int64_t cap_tasks);
 

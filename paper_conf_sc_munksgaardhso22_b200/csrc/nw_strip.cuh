@@ -204,6 +204,7 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
   const bool tracing = P.trace != nullptr;
   long long ev_cyc = 0, spin_cyc = 0, wait_cyc = 0;  // debug cycle accounting (trace only)
   long long blk_cyc = 0;                              // steady-state step blocks
+  long long ph_cyc[5] = {0, 0, 0, 0, 0};              // event sub-phases (trace only)
 
   const uint32_t s_prog = smem_u32(smem + 8);
   const uint32_t s_bring = smem_u32(smem + 128);
@@ -464,9 +465,13 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
       if (tracing) wait_cyc += clock64() - c_w0;
     }
     // event Q reached: score chunk Q-STORE_DELAY is complete, ref chunk Q-SKEW-1 no longer read
+    const long long c_p1 = tracing ? clock64() : 0;
+    if (tracing) ph_cyc[0] += c_p1 - c_ev0;
     rvn_valid = false;  // rows of the new chunk may be read only after this event's check
     __syncwarp();
     if (t == 0 && !(P.dbg_skip & 4u)) mbar_arrive(bar_ev + 8 * (Q % C::SLOTS));
+    const long long c_p2 = tracing ? clock64() : 0;
+    if (tracing) ph_cyc[1] += c_p2 - c_p1;
     if (sig0 >= nsteps) {
       if (tracing) ev_cyc += clock64() - c_ev0;
       continue;
@@ -481,6 +486,8 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
       __syncwarp();
       prefetch_block(Q + D);  // into the slot of block Q+D-4, consumed two events ago
     }
+    const long long c_p3 = tracing ? clock64() : 0;
+    if (tracing) ph_cyc[2] += c_p3 - c_p2;
     if (src != kSrcPlain && !(P.dbg_skip & 8u)) {
       // the block needs rows sig0+1 .. sig0+CH of the left border (lanes 0 .. CH-1)
       auto ready = [&]() {
@@ -499,6 +506,8 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
         spin_cyc += clock64() - c_0;
       }
     }
+    const long long c_p4 = tracing ? clock64() : 0;
+    if (tracing) ph_cyc[3] += c_p4 - c_p3;
     if constexpr (SINK == kSinkSmem) {
       // back-pressure: rows written in this block are <= sig0+CH-31; their ring slots must hold
       // rows the consumer (warp w+1) already consumed
@@ -509,7 +518,11 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
           if (globaltimer_ns() - t0 > P.spin_limit_ns) watchdog_trap(P.err);
       }
     }
-    if (tracing) ev_cyc += clock64() - c_ev0;
+    if (tracing) {
+      const long long c_p5 = clock64();
+      ph_cyc[4] += c_p5 - c_p4;
+      ev_cyc += c_p5 - c_ev0;
+    }
     // ---- CH wavefront steps: lane t computes row sig+1-t, columns c0+tK .. c0+tK+K-1
     if (sig0 >= 31 && sig0 + CH <= n) {  // steady state: all 32 lanes on rows 1..n
       const long long c_b0 = tracing ? clock64() : 0;
@@ -538,6 +551,8 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
     e[5] = static_cast<unsigned long long>(wait_cyc);  // of which: waits on the staging warp
     e[6] = static_cast<unsigned long long>(spin_cyc);  // of which: left-border spins
     e[7] = static_cast<unsigned long long>(clock64() - c_task0);
+    if (P.trace2 != nullptr)
+      for (int k = 0; k < 5; ++k) P.trace2[8 * task + 2 + k] = static_cast<unsigned long long>(ph_cyc[k]);
   }
 }
 
@@ -748,8 +763,8 @@ __device__ __forceinline__ void nw_stage(const StripParams& P, const long long t
   }
   cbase += static_cast<uint32_t>(nch);
   if (P.trace2 != nullptr && t == 0 && task < P.trace_cap) {
-    P.trace2[2 * task] = static_cast<unsigned long long>(clock64() - c_task0);
-    P.trace2[2 * task + 1] = static_cast<unsigned long long>(wait_cyc);
+    P.trace2[8 * task] = static_cast<unsigned long long>(clock64() - c_task0);
+    P.trace2[8 * task + 1] = static_cast<unsigned long long>(wait_cyc);
   }
 }
 
