@@ -345,6 +345,8 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
   }
   const uint32_t* const profp = prof + t;
   uint32_t tok = 0;  // produced by each chunk's mbarrier wait, consumed by the ref loads
+  uint64_t st_cache = 0;  // last staging progress word read (acquired) by this warp
+  int bp_cache = 0;       // last consumer progress read (back-pressure)
   int negp[K];       // -(m+1) p
 #pragma unroll
   for (int m = 0; m < K; ++m) negp[m] = -(m + 1) * p;
@@ -447,11 +449,14 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
       const long long c_w0 = tracing ? clock64() : 0;
       const uint32_t need_rd = cbase + static_cast<uint32_t>(Q) + 1u;
       const uint32_t need_st = Q >= C::SLOTS ? cbase + static_cast<uint32_t>(Q - C::SLOTS) + 1u : 0u;
-      uint64_t stt = ld_acquire_cta(s_state);
       auto ok = [&](uint64_t v) {
         return (SEQ || static_cast<int>(static_cast<uint32_t>(v) - need_rd) >= 0) &&
                static_cast<int>(static_cast<uint32_t>(v >> 32) - need_st) >= 0;
       };
+      // the last progress word seen usually still covers this event (the staging warp runs
+      // LOOKW chunks ahead): re-read it only when it does not
+      uint64_t stt = st_cache;
+      if (!ok(stt)) stt = ld_acquire_cta(s_state);
       if (!ok(stt)) {
         const uint64_t t0 = globaltimer_ns();
         unsigned spins = 0;
@@ -460,6 +465,7 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
           if ((++spins & 1023u) == 0 && globaltimer_ns() - t0 > P.spin_limit_ns) watchdog_trap(P.err);
         } while (!ok(stt));
       }
+      st_cache = stt;
       // token (always 0) data-dependent on the acquire: the ref loads cannot move above it
       asm volatile("and.b32 %0, %1, 0;" : "=r"(tok) : "r"(static_cast<uint32_t>(stt)));
       if (tracing) wait_cyc += clock64() - c_w0;
@@ -512,9 +518,9 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
       // back-pressure: rows written in this block are <= sig0+CH-31; their ring slots must hold
       // rows the consumer (warp w+1) already consumed
       const int rmax = sig0 + CH - 31;
-      if (rmax - kBR > 0 && rmax - kBR > lds32_volatile(prog_out)) {
+      if (rmax - kBR > bp_cache && rmax - kBR > (bp_cache = lds32_volatile(prog_out))) {
         const uint64_t t0 = globaltimer_ns();
-        while (rmax - kBR > lds32_volatile(prog_out))
+        while (rmax - kBR > (bp_cache = lds32_volatile(prog_out)))
           if (globaltimer_ns() - t0 > P.spin_limit_ns) watchdog_trap(P.err);
       }
     }
@@ -740,26 +746,33 @@ __device__ __forceinline__ void nw_stage(const StripParams& P, const long long t
     if constexpr (!SEQ) {
       if (Q + C::LOOKW < nch) issue_ref(Q + C::LOOKW);
       cp_async_commit();
-      // warm L2 with the ref rows kPF chunks further ahead: one 128-byte line per lane
+      // warm L2 with the ref rows kPF chunks further ahead (every 128-byte line of each row)
       const int cp = Q + C::LOOKW + kPF;
       if (cp < nch) {
-        const int i = t / 4, ln = t % 4;
-        const int r = cp * CH + 1 + i;
-        const uintptr_t g = reinterpret_cast<uintptr_t>(R + static_cast<long long>(r) * P.ldr + c0) + 128u * ln;
-        prefetch_l2_p(i < CH && r <= n && 128 * ln < 4 * ws + 128, reinterpret_cast<const void*>(g));
+        constexpr int LINES = (4 * C::W + 8 + 127) / 128 + 1;  // lines touched by one row segment
+#pragma unroll
+        for (int it = 0; it < (CH * LINES + 31) / 32; ++it) {
+          const int f = t + 32 * it;
+          const int i = f / LINES, ln = f - (f / LINES) * LINES;
+          const int r = cp * CH + 1 + i;
+          const uintptr_t g0 = reinterpret_cast<uintptr_t>(R + static_cast<long long>(r) * P.ldr + c0) & ~static_cast<uintptr_t>(127);
+          prefetch_l2_p(i < CH && r <= n, reinterpret_cast<const void*>(g0 + 128u * ln));
+        }
       }
+    }
+    if constexpr (!SEQ) {
+      cp_async_wait<C::LOOKW - 1>();  // chunks <= Q+1 landed: publish before the stores
+      rd = cbase + static_cast<uint32_t>(min(Q + 2, nch));
+      __syncwarp();
+      if (t == 0) st_release_cta_v2(s_state, rd, sd);
     }
     const int cs = Q - C::STORE_DELAY;
     if (cs >= 0 && cs < nch) {
       store_sc(cs);
       sd = cbase + static_cast<uint32_t>(cs) + 1u;
+      __syncwarp();  // every lane's stores of this chunk read their slots
+      if (t == 0) st_release_cta_v2(s_state, rd, sd);
     }
-    if constexpr (!SEQ) {
-      cp_async_wait<C::LOOKW - 1>();  // chunks <= Q+1 landed
-      rd = cbase + static_cast<uint32_t>(min(Q + 2, nch));
-    }
-    __syncwarp();  // every lane's copies / stores of this iteration are done
-    if (t == 0) st_release_cta_v2(s_state, rd, sd);
   }
   cbase += static_cast<uint32_t>(nch);
   if (P.trace2 != nullptr && t == 0 && task < P.trace_cap) {
