@@ -47,37 +47,41 @@ namespace nwb200 {
 
 constexpr int kBarBytes = 1024;  // per band pair: ev mbarriers [128,256), progress word [384], border prefetch ring [512,1024)
 constexpr int kBR = 256;      // shared border ring entries between consecutive warps of a CTA
-constexpr int kRing = 64;     // rows per staging ring (power of two)
+constexpr int kNEv = 16;      // event mbarrier slots (compute leads staging by <= 2 events)
 constexpr int kPF = 4;        // ref chunks prefetched into L2 beyond the smem lookahead
 constexpr unsigned kErrWatchdog = 0xBADB0001u;
 
 // Geometry of one kernel instance.  Events happen every CH steps (event Q starts step CH*Q).
 // In block Q lane t touches rows CH*Q+1-t .. CH*Q+CH-t: chunks Q-SKEW .. Q (the 31-row skew).
-template <int K_, bool SEQ_, int NW_, int CH_, int LOOK_>
+template <int K_, bool SEQ_, int NW_, int CH_, int RR_, int SR_>
 struct StripCfg {
-  static constexpr int K = K_, NW = NW_, CH = CH_, LOOK = LOOK_;
+  static constexpr int K = K_, NW = NW_, CH = CH_;
   static constexpr bool SEQ = SEQ_;
   static constexpr int W = 32 * K;   // warp band width (columns)
   static constexpr int RS = W + 36;  // row slot (words): W + 3 head + 3 tail + 28 swizzle, 16B multiple
   static constexpr int SKEW = (31 + CH - 1) / CH;
-  static constexpr int SLOTS = kRing / CH;           // chunks per ring
-  static constexpr int STORE_DELAY = SKEW + 1;       // chunk c complete after step CH*c+CH-1+31
-  static constexpr int MAXR = W / 4 + 2;             // 16-byte chunks of a ref row superset
-  static constexpr int MAXS = W / 4;                 // 16-byte chunks of a score row interior
+  static constexpr int RR = SEQ ? CH : RR_;           // ref ring rows
+  static constexpr int SR = SR_;                      // score ring rows
+  static constexpr int REF_SLOTS = RR / CH;           // ref chunks per ring
+  static constexpr int SLOTS = SR / CH;               // score chunks per ring
+  static constexpr int STORE_DELAY = SKEW + 1;        // chunk c complete after step CH*c+CH-1+31
+  static constexpr int LOOKW = REF_SLOTS - SKEW - 1;  // ref chunks the staging warp runs ahead
+  static constexpr int MAXR = W / 4 + 2;              // 16-byte chunks of a ref row superset
+  static constexpr int MAXS = W / 4;                  // 16-byte chunks of a score row interior
   static constexpr int ITER_R = (CH * MAXR + 31) / 32;
   static constexpr int ITER_S = (CH * MAXS + 31) / 32;
-  static constexpr int REF_ROWS = SEQ ? 0 : kRing;
+  static constexpr int REF_ROWS = SEQ ? 0 : RR;
   static constexpr int PROF_WORDS = SEQ ? 32 * 32 : 0;
-  static constexpr size_t kWarpSmem = kBarBytes + 4ull * ((size_t)REF_ROWS * RS + (size_t)kRing * RS + PROF_WORDS);
+  static constexpr size_t kWarpSmem = kBarBytes + 4ull * ((size_t)REF_ROWS * RS + (size_t)SR * RS + PROF_WORDS);
   static constexpr size_t kCtaHdr = 128 + (size_t)(NW - 1) * kBR * 8;
   static constexpr size_t kSmem = kCtaHdr + NW * kWarpSmem;
   static_assert(32 % CH == 0 && 2 * CH <= 32, "events must align with the 32-row border windows");
-  static_assert(LOOK + SKEW + 1 <= SLOTS, "ref ring too small for the lookahead");
-  static_assert(STORE_DELAY + 1 <= SLOTS, "score ring too small for the store delay");
+  static_assert(RR % CH == 0 && SR % CH == 0, "rings hold whole chunks");
+  static_assert(SEQ || LOOKW >= 1, "ref ring too small for any lookahead");
+  static_assert(SLOTS >= STORE_DELAY + 1, "score ring too small for the store delay");
   static_assert(RS % 4 == 0 && kWarpSmem % 16 == 0, "16-byte aligned rings");
-  static_assert(((size_t)kRing * RS) % 32 == 0, "ring wrap keeps banks");
-  static_assert(NW <= 8 && SLOTS <= 16, "header / barrier space");
-  static constexpr int LOOKW = SLOTS - SKEW - 1;     // ref chunks the staging warp runs ahead
+  static_assert(((size_t)RR * RS) % 32 == 0 && ((size_t)SR * RS) % 32 == 0, "ring wrap keeps banks");
+  static_assert(NW <= 8, "header space");
 };
 
 // ---- the schedule (shared by the kernel and the host export nw_strip_map, pin P7) --------
@@ -211,7 +215,7 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
   const uint32_t bar_ev = smem_u32(wsm) + 128, s_state = smem_u32(wsm) + 384;
   int32_t* const ref_ring = reinterpret_cast<int32_t*>(wsm + kBarBytes);
   int32_t* const sc_ring = ref_ring + C::REF_ROWS * RS;
-  uint32_t* const prof = reinterpret_cast<uint32_t*>(sc_ring + kRing * RS);
+  uint32_t* const prof = reinterpret_cast<uint32_t*>(sc_ring + C::SR * RS);
 
   const int n = static_cast<int>(P.n);
   const int nch = (n + CH - 1) / CH;
@@ -314,7 +318,8 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
     for (int q = 0; q < D; ++q) prefetch_block(q);
   // per-lane ring addressing: row r (= step + 1 - t) lives at ring row (r-1) & 63
   const int r0 = 1 - t;
-  int rr = r0 - 1;  // r - 1
+  int rowR = (((r0 - 1) % C::RR) + C::RR) % C::RR;  // ring rows of this lane's current row
+  int rowS = (((r0 - 1) % C::SR) + C::SR) % C::SR;
   int gR = static_cast<int>((GR0 + static_cast<uintptr_t>(static_cast<intptr_t>(r0) * P.ldr)) & 31);
   int gS = static_cast<int>((GS0 + static_cast<uintptr_t>(static_cast<intptr_t>(r0) * P.lds)) & 31);
   const int ldr32 = static_cast<int>(P.ldr & 31), lds32 = static_cast<int>(P.lds & 31);
@@ -322,8 +327,8 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
   // right-border publish (lane out_lane holds the band's last column in Pv[K-1]; every band
   // with a right neighbour is full width)
   const bool do_out = t == out_lane;
-  uint64_t* gout = lout != nullptr ? lout + r0 : nullptr;
-  uint32_t sout_hi = lout_tag + static_cast<uint32_t>(r0);
+  uint32_t sout_hi = (SINK == kSinkSmem ? lout_tag : 0u) + static_cast<uint32_t>(r0);  // tag | row (row for global)
+  const uint32_t gstage = smem_u32(wsm);  // [2*CH] x 8 bytes: global-sink entries awaiting publish
   // SEQ: per-band substitution profile prof[x][t] = pack_m subst[x][b[c0-1+tK+m]] (int8 x K)
   const uint8_t* const A = SEQ ? P.seq_a + pair * P.psa : nullptr;
   int a0 = 0, a1 = 0;  // residues of this lane's current and next row (software pipeline)
@@ -360,7 +365,7 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
       (void)rr_;
       (void)gR_;
     } else {
-      const uint32_t aR = laneR + 4u * RS * static_cast<uint32_t>(rr_ & (kRing - 1)) + 4u * static_cast<uint32_t>(gR_ & 31);
+      const uint32_t aR = laneR + 4u * RS * static_cast<uint32_t>(rr_) + 4u * static_cast<uint32_t>(gR_ & 31);
 #pragma unroll
       for (int m = 0; m < K; ++m) out[m] = lds_tok(aR + 4 * m, tok);
     }
@@ -372,17 +377,18 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
   // one wavefront step; ALL = every lane's row is in 1..n (steady state, no predicates)
   auto step = [&](const int sig, auto all_tag) {
     constexpr bool ALL = decltype(all_tag)::value;
-    const uint32_t roff = 4u * RS * static_cast<uint32_t>(rr & (kRing - 1));
+    const int rowR1 = rowR + 1 == C::RR ? 0 : rowR + 1;  // ring row of the next row
+    const uint32_t soff = 4u * RS * static_cast<uint32_t>(rowS);
     int rv[K];
     if constexpr (SEQ) {
       const uint32_t pw = profp[32 * a0];
 #pragma unroll
       for (int m = 0; m < K; ++m) rv[m] = prmt_sext(pw, 0x8880u + 0x1111u * m);  // sign-extended byte m
     } else {
-      if (!rvn_valid) load_ref(rvn, rr, gR);
+      if (!rvn_valid) load_ref(rvn, rowR, gR);
 #pragma unroll
       for (int m = 0; m < K; ++m) rv[m] = rvn[m];
-      load_ref(rvn, rr + 1, gR + ldr32);  // next row (same chunk block or ring-resident)
+      load_ref(rvn, rowR1, gR + ldr32);  // next row (same chunk block or ring-resident)
       rvn_valid = true;
     }
     const int bval = __shfl_sync(FULL, static_cast<int>(static_cast<uint32_t>(cur)), sig & (CH - 1));  // lane 0's left
@@ -412,15 +418,15 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
 #pragma unroll
       for (int m = 0; m < K; ++m) Pv[m] = __viaddmax_s32(L, negp[m], Y[m]);  // max(L - (m+1)p, Y_m)
       Lprev = L;
-      const uint32_t aS = laneS + roff + 4u * static_cast<uint32_t>(gS & 31);
+      const uint32_t aS = laneS + soff + 4u * static_cast<uint32_t>(gS & 31);
 #pragma unroll
       for (int m = 0; m < K; ++m) sts_s32(aS + 4 * m, Pv[m]);
       const uint32_t vo = static_cast<uint32_t>(Pv[K - 1]);
       if constexpr (SINK == kSinkSmem) {
         st_entry_smem(do_out, bring_out + 8u * (sout_hi & (kBR - 1)), vo, sout_hi);
       } else if constexpr (SINK == kSinkGlobal) {
-        st_entry_gpu(do_out && !lout_sys, gout, vo, lout_tag);
-        st_entry_sys(do_out && lout_sys, gout, vo, lout_tag);
+        // staged in shared memory, published CH rows at a time at the next event
+        st_entry_smem(do_out, gstage + 8u * (sout_hi & (2 * CH - 1)), vo, 0u);
       } else {
         (void)vo;
       }
@@ -431,11 +437,11 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
       a0 = a1;
       a1 = __ldg(A + min(max(lane_row(sig, t) + 1, 0), n - 1)) & 31;  // residue of row r+2
     }
-    ++rr;
+    rowR = rowR1;
+    rowS = rowS + 1 == C::SR ? 0 : rowS + 1;
     gR += ldr32;
     gS += lds32;
-    if constexpr (SINK == kSinkGlobal) ++gout;
-    if constexpr (SINK == kSinkSmem) ++sout_hi;
+    if constexpr (SINK != kSinkNone) ++sout_hi;
   };
 
   for (int Q = 0; Q <= nch + C::STORE_DELAY - 1; ++Q) {
@@ -475,9 +481,20 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
     if (tracing) ph_cyc[0] += c_p1 - c_ev0;
     rvn_valid = false;  // rows of the new chunk may be read only after this event's check
     __syncwarp();
-    if (t == 0 && !(P.dbg_skip & 4u)) mbar_arrive(bar_ev + 8 * (Q % C::SLOTS));
+    if (t == 0 && !(P.dbg_skip & 4u)) mbar_arrive(bar_ev + 8 * (Q % kNEv));
     const long long c_p2 = tracing ? clock64() : 0;
     if (tracing) ph_cyc[1] += c_p2 - c_p1;
+    if constexpr (SINK == kSinkGlobal) {
+      // publish the rows the out lane finished during block Q-1 (rows CH*(Q-1)+1-out_lane ..
+      // CH*Q-out_lane), CH entries at once
+      if (Q > 0) {
+        const int row = CH * (Q - 1) + 1 - out_lane + t;
+        const bool go = t < CH && row >= 1 && row <= n;
+        const uint32_t v = go ? static_cast<uint32_t>(lds64_volatile(gstage + 8u * (row & (2 * CH - 1)))) : 0u;
+        st_entry_gpu(go && !lout_sys, lout + row, v, lout_tag);
+        st_entry_sys(go && lout_sys, lout + row, v, lout_tag);
+      }
+    }
     if (sig0 >= nsteps) {
       if (tracing) ev_cyc += clock64() - c_ev0;
       continue;
@@ -623,7 +640,7 @@ __device__ __forceinline__ void nw_stage(const StripParams& P, const long long t
   // then every lane arrives on the chunk's mbarrier when its copies have landed.
   auto issue_ref = [&](int c) {
     const uintptr_t cb = static_cast<uintptr_t>(c) * rstride;
-    const uint32_t db = refR0 + 4u * ((c * CH) & (kRing - 1)) * RS;
+    const uint32_t db = refR0 + 4u * ((c * CH) % C::RR) * RS;
     const int Dc = (c * rDc) & 31;
     const int rlim = n - c * CH;  // row i valid iff i < rlim
     if (!(last_band && c == last_chunk)) {
@@ -695,7 +712,7 @@ __device__ __forceinline__ void nw_stage(const StripParams& P, const long long t
 
   auto store_sc = [&](int c) {
     const uintptr_t cb = static_cast<uintptr_t>(c) * sstride;
-    const uint32_t sb = scR0 + 4u * ((c * CH) & (kRing - 1)) * RS;
+    const uint32_t sb = scR0 + 4u * ((c * CH) % C::SR) * RS;
     const int Dc = (c * sDc) & 31;
     const int rlim = n - c * CH;
     int4 v[C::ITER_S];
@@ -738,7 +755,7 @@ __device__ __forceinline__ void nw_stage(const StripParams& P, const long long t
   __syncwarp();
   if (t == 0) st_release_cta_v2(s_state, rd, sd);
   for (int Q = 0; Q <= nch + C::STORE_DELAY - 1; ++Q) {
-    const int sl = Q % C::SLOTS;
+    const int sl = Q % kNEv;
     const long long c_w0 = clock64();
     mbar_wait(bar_ev + 8 * sl, (ph_ev >> sl) & 1u);
     ph_ev ^= 1u << sl;
@@ -795,7 +812,7 @@ __global__ void __launch_bounds__(64 * C::NW, 1) nw_strip_kernel(const __grid_co
   unsigned char* const wsm = smem + C::kCtaHdr + w * C::kWarpSmem;
   if (!staging && t == 0) {
     const uint32_t b = smem_u32(wsm);
-    for (int i = 0; i < C::SLOTS; ++i) mbar_init(b + 128 + 8 * i, 1);  // ev: the compute warp reached an event
+    for (int i = 0; i < kNEv; ++i) mbar_init(b + 128 + 8 * i, 1);  // ev: the compute warp reached an event
     st_release_cta_v2(b + 384, 0u, 0u);                                 // staging progress word
   }
   fence_mbar_init();
