@@ -196,10 +196,10 @@ enum : int { kSinkNone = 0, kSinkSmem = 1, kSinkGlobal = 2 };
 
 // One band (task) of the persistent kernel; SINK is specialised so the steady-state step has no
 // branches.
-template <class C, int SINK>
+template <class C>
 __device__ __forceinline__ void nw_band(const StripParams& P, const long long task, const int w, const int t,
                                         unsigned char* const smem, unsigned char* const wsm, const uint32_t gen,
-                                        uint32_t& cbase) {
+                                        uint32_t& cbase, const int SINK) {
   constexpr int K = C::K, RS = C::RS, CH = C::CH;
   constexpr bool SEQ = C::SEQ;
   constexpr unsigned FULL = 0xffffffffu;
@@ -250,7 +250,7 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
   uint64_t* lout = nullptr;
   uint32_t lout_tag = 0;
   bool lout_sys = false;
-  if constexpr (SINK == kSinkGlobal) {
+  if (SINK == kSinkGlobal) {
     if (last_band) {
       lout = P.halo_out;
       lout_tag = P.halo_epoch;
@@ -259,7 +259,7 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
       lout = P.xbuf + (pair * (P.nbands - 1) + band) * xstride(n);
       lout_tag = P.epoch;
     }
-  } else if constexpr (SINK == kSinkSmem) {
+  } else if (SINK == kSinkSmem) {
     lout_tag = gen;
   }
   const uint32_t bring_in = s_bring + (w - 1) * kBR * 8;   // src == kSrcSmem
@@ -326,9 +326,11 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
   const uint32_t laneR = refR0 + 4u * t * K, laneS = scR0 + 4u * t * K;
   // right-border publish (lane out_lane holds the band's last column in Pv[K-1]; every band
   // with a right neighbour is full width)
-  const bool do_out = t == out_lane;
+  const bool do_out = t == out_lane && SINK != kSinkNone;
   uint32_t sout_hi = (SINK == kSinkSmem ? lout_tag : 0u) + static_cast<uint32_t>(r0);  // tag | row (row for global)
   const uint32_t gstage = smem_u32(wsm);  // [2*CH] x 8 bytes: global-sink entries awaiting publish
+  const uint32_t out_base = SINK == kSinkSmem ? bring_out : gstage;
+  const uint32_t out_mask = SINK == kSinkSmem ? kBR - 1 : 2 * CH - 1;
   // SEQ: per-band substitution profile prof[x][t] = pack_m subst[x][b[c0-1+tK+m]] (int8 x K)
   const uint8_t* const A = SEQ ? P.seq_a + pair * P.psa : nullptr;
   int a0 = 0, a1 = 0;  // residues of this lane's current and next row (software pipeline)
@@ -421,15 +423,9 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
       const uint32_t aS = laneS + soff + 4u * static_cast<uint32_t>(gS & 31);
 #pragma unroll
       for (int m = 0; m < K; ++m) sts_s32(aS + 4 * m, Pv[m]);
-      const uint32_t vo = static_cast<uint32_t>(Pv[K - 1]);
-      if constexpr (SINK == kSinkSmem) {
-        st_entry_smem(do_out, bring_out + 8u * (sout_hi & (kBR - 1)), vo, sout_hi);
-      } else if constexpr (SINK == kSinkGlobal) {
-        // staged in shared memory, published CH rows at a time at the next event
-        st_entry_smem(do_out, gstage + 8u * (sout_hi & (2 * CH - 1)), vo, 0u);
-      } else {
-        (void)vo;
-      }
+      // publish the band's last column (lane out_lane, Pv[K-1]): straight into warp w+1's
+      // shared ring, or into the local staging ring flushed to global memory at each event
+      st_entry_smem(do_out, out_base + 8u * (sout_hi & out_mask), static_cast<uint32_t>(Pv[K - 1]), sout_hi);
     }
     vlast = Pv[K - 1];
     // advance this lane to row r+1
@@ -441,7 +437,7 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
     rowS = rowS + 1 == C::SR ? 0 : rowS + 1;
     gR += ldr32;
     gS += lds32;
-    if constexpr (SINK != kSinkNone) ++sout_hi;
+    ++sout_hi;
   };
 
   for (int Q = 0; Q <= nch + C::STORE_DELAY - 1; ++Q) {
@@ -484,7 +480,7 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
     if (t == 0 && !(P.dbg_skip & 4u)) mbar_arrive(bar_ev + 8 * (Q % kNEv));
     const long long c_p2 = tracing ? clock64() : 0;
     if (tracing) ph_cyc[1] += c_p2 - c_p1;
-    if constexpr (SINK == kSinkGlobal) {
+    if (SINK == kSinkGlobal) {
       // publish the rows the out lane finished during block Q-1 (rows CH*(Q-1)+1-out_lane ..
       // CH*Q-out_lane), CH entries at once
       if (Q > 0) {
@@ -531,7 +527,7 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
     }
     const long long c_p4 = tracing ? clock64() : 0;
     if (tracing) ph_cyc[3] += c_p4 - c_p3;
-    if constexpr (SINK == kSinkSmem) {
+    if (SINK == kSinkSmem) {
       // back-pressure: rows written in this block are <= sig0+CH-31; their ring slots must hold
       // rows the consumer (warp w+1) already consumed
       const int rmax = sig0 + CH - 31;
@@ -842,12 +838,7 @@ __global__ void __launch_bounds__(64 * C::NW, 1) nw_strip_kernel(const __grid_co
           sink = P.halo_out ? kSinkGlobal : kSinkNone;
         else
           sink = (w < NW - 1) ? kSinkSmem : kSinkGlobal;
-        if (sink == kSinkSmem)
-          nw_band<C, kSinkSmem>(P, task, w, t, smem, wsm, gen, cbase);
-        else if (sink == kSinkGlobal)
-          nw_band<C, kSinkGlobal>(P, task, w, t, smem, wsm, gen, cbase);
-        else
-          nw_band<C, kSinkNone>(P, task, w, t, smem, wsm, gen, cbase);
+        nw_band<C>(P, task, w, t, smem, wsm, gen, cbase, sink);
       }
     }
     __syncthreads();  // group end: every warp done (shared border rings / progress reusable)
