@@ -67,8 +67,8 @@ nw_status check_range(int64_t n, int32_t p) {
 // LOOK chunks of ref prefetch (DESIGN.md §4.3 sizes the rings).
 using CfgK2 = StripCfg<2, false, 4, 8, 64, 48>;
 using CfgK2S = StripCfg<2, true, 4, 8, 64, 48>;
-using CfgK4 = StripCfg<4, false, 2, 8, 96, 48>;
-using CfgK4S = StripCfg<4, true, 2, 8, 96, 48>;
+using CfgK4 = StripCfg<4, false, 2, 16, 96, 64>;
+using CfgK4S = StripCfg<4, true, 2, 16, 96, 64>;
 
 struct DevInfo {
   bool init = false;

@@ -45,7 +45,10 @@
 
 namespace nwb200 {
 
-constexpr int kBarBytes = 1024;  // per band pair: ev mbarriers [128,256), progress word [384], border prefetch ring [512,1024)
+// per band pair header: ev mbarriers [0,128), progress word [128], global-sink staging ring
+// [256,512), border prefetch ring [512,1280)
+constexpr int kBarBytes = 2048;
+constexpr int kHdrEv = 0, kHdrState = 128, kHdrGstage = 256, kHdrBpre = 512;
 constexpr int kBR = 256;      // shared border ring entries between consecutive warps of a CTA
 constexpr int kNEv = 16;      // event mbarrier slots (compute leads staging by <= 2 events)
 constexpr int kPF = 4;        // ref chunks prefetched into L2 beyond the smem lookahead
@@ -75,13 +78,14 @@ struct StripCfg {
   static constexpr size_t kWarpSmem = kBarBytes + 4ull * ((size_t)REF_ROWS * RS + (size_t)SR * RS + PROF_WORDS);
   static constexpr size_t kCtaHdr = 128 + (size_t)(NW - 1) * kBR * 8;
   static constexpr size_t kSmem = kCtaHdr + NW * kWarpSmem;
-  static_assert(32 % CH == 0 && 2 * CH <= 32, "events must align with the 32-row border windows");
+  static_assert(32 % CH == 0 && CH <= 16, "events must align with the 32-row border windows");
   static_assert(RR % CH == 0 && SR % CH == 0, "rings hold whole chunks");
   static_assert(SEQ || LOOKW >= 1, "ref ring too small for any lookahead");
   static_assert(SLOTS >= STORE_DELAY + 1, "score ring too small for the store delay");
   static_assert(RS % 4 == 0 && kWarpSmem % 16 == 0, "16-byte aligned rings");
   static_assert(((size_t)RR * RS) % 32 == 0 && ((size_t)SR * RS) % 32 == 0, "ring wrap keeps banks");
   static_assert(NW <= 8, "header space");
+  static_assert(2 * CH * 8 <= 256 && 4 * (CH + 2) * 8 <= 768, "per-band header regions");
 };
 
 // ---- the schedule (shared by the kernel and the host export nw_strip_map, pin P7) --------
@@ -212,7 +216,7 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
 
   const uint32_t s_prog = smem_u32(smem + 8);
   const uint32_t s_bring = smem_u32(smem + 128);
-  const uint32_t bar_ev = smem_u32(wsm) + 128, s_state = smem_u32(wsm) + 384;
+  const uint32_t bar_ev = smem_u32(wsm) + kHdrEv, s_state = smem_u32(wsm) + kHdrState;
   int32_t* const ref_ring = reinterpret_cast<int32_t*>(wsm + kBarBytes);
   int32_t* const sc_ring = ref_ring + C::REF_ROWS * RS;
   uint32_t* const prof = reinterpret_cast<uint32_t*>(sc_ring + C::SR * RS);
@@ -300,7 +304,7 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
   // directly at the event.  Ring slot of block q: entries of rows CH*q .. CH*q+CH+1.
   constexpr int D = 2;
   constexpr uint32_t kSlotB = 8u * (CH + 2);
-  const uint32_t bpre = smem_u32(wsm) + 512;
+  const uint32_t bpre = smem_u32(wsm) + kHdrBpre;
   auto prefetch_block = [&](int q) {  // block q = rows CH*q+1 .. CH*q+CH
     const uint32_t slot = bpre + kSlotB * static_cast<uint32_t>(q & 3);
     if (src == kSrcGlobal) {
@@ -328,7 +332,7 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
   // with a right neighbour is full width)
   const bool do_out = t == out_lane && SINK != kSinkNone;
   uint32_t sout_hi = (SINK == kSinkSmem ? lout_tag : 0u) + static_cast<uint32_t>(r0);  // tag | row (row for global)
-  const uint32_t gstage = smem_u32(wsm);  // [2*CH] x 8 bytes: global-sink entries awaiting publish
+  const uint32_t gstage = smem_u32(wsm) + kHdrGstage;  // [2*CH] x 8 bytes: global-sink entries awaiting publish
   const uint32_t out_base = SINK == kSinkSmem ? bring_out : gstage;
   const uint32_t out_mask = SINK == kSinkSmem ? kBR - 1 : 2 * CH - 1;
   // SEQ: per-band substitution profile prof[x][t] = pack_m subst[x][b[c0-1+tK+m]] (int8 x K)
@@ -585,7 +589,7 @@ __device__ __forceinline__ void nw_stage(const StripParams& P, const long long t
   constexpr bool SEQ = C::SEQ;
   const long long c_task0 = clock64();
   long long wait_cyc = 0;
-  const uint32_t bar_ev = smem_u32(wsm) + 128, s_state = smem_u32(wsm) + 384;
+  const uint32_t bar_ev = smem_u32(wsm) + kHdrEv, s_state = smem_u32(wsm) + kHdrState;
   int32_t* const ref_ring = reinterpret_cast<int32_t*>(wsm + kBarBytes);
   int32_t* const sc_ring = ref_ring + C::REF_ROWS * RS;
   const int n = static_cast<int>(P.n);
@@ -808,8 +812,8 @@ __global__ void __launch_bounds__(64 * C::NW, 1) nw_strip_kernel(const __grid_co
   unsigned char* const wsm = smem + C::kCtaHdr + w * C::kWarpSmem;
   if (!staging && t == 0) {
     const uint32_t b = smem_u32(wsm);
-    for (int i = 0; i < kNEv; ++i) mbar_init(b + 128 + 8 * i, 1);  // ev: the compute warp reached an event
-    st_release_cta_v2(b + 384, 0u, 0u);                                 // staging progress word
+    for (int i = 0; i < kNEv; ++i) mbar_init(b + kHdrEv + 8 * i, 1);  // ev: the compute warp reached an event
+    st_release_cta_v2(b + kHdrState, 0u, 0u);                            // staging progress word
   }
   fence_mbar_init();
   // shared border rings start invalid (tag 0xFFFFFFFF never equals gen | row, row < 2^30)
