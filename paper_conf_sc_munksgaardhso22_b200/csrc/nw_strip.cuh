@@ -549,7 +549,8 @@ __device__ __forceinline__ void nw_band(const StripParams& P, const long long ta
     // ---- CH wavefront steps: lane t computes row sig+1-t, columns c0+tK .. c0+tK+K-1
     if (sig0 >= 31 && sig0 + CH <= n) {  // steady state: all 32 lanes on rows 1..n
       const long long c_b0 = tracing ? clock64() : 0;
-#pragma unroll
+      // 4-step unrolled body: keeps the hot loop inside the L0 instruction cache
+#pragma unroll 4
       for (int j = 0; j < CH; ++j) step(sig0 + j, std::true_type{});
       if (tracing) blk_cyc += clock64() - c_b0;
     } else {
