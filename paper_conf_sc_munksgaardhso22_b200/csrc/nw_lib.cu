@@ -15,6 +15,7 @@
 #include "nw.h"
 #include "nw_diag.cuh"
 #include "nw_strip.cuh"
+#include "nw_wave.cuh"
 
 using namespace nwb200;
 
@@ -69,11 +70,25 @@ using CfgK2 = StripCfg<2, false, 4, 8, 64, 48>;
 using CfgK2S = StripCfg<2, true, 4, 8, 64, 48>;
 using CfgK4 = StripCfg<4, false, 2, 16, 96, 64>;
 using CfgK4S = StripCfg<4, true, 2, 16, 96, 64>;
+// v5 self-staging wavefront kernels (nw_wave.cuh)
+using WCfgK2 = WaveCfg<2, false, 4>;
+using WCfgK2S = WaveCfg<2, true, 4>;
+using WCfgK4 = WaveCfg<4, false, 2>;
+using WCfgK4S = WaveCfg<4, true, 2>;
+
+bool use_wave() {
+  static const bool v = [] {
+    const char* e = std::getenv("NW_KERNEL");
+    return !(e && e[0] == 's');  // NW_KERNEL=strip selects the v4 kernel (A/B only)
+  }();
+  return v;
+}
 
 struct DevInfo {
   bool init = false;
   int sms = 0;
   int occ[2][2] = {{0, 0}, {0, 0}};  // [K==4][SEQ]
+  int wocc[2][2] = {{0, 0}, {0, 0}};
 };
 
 template <class C>
@@ -82,6 +97,14 @@ cudaError_t setup_kernel(int* occ) {
                                        static_cast<int>(C::kSmem));
   if (e != cudaSuccess) return e;
   return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, nw_strip_kernel<C>, 64 * C::NW, C::kSmem);
+}
+
+template <class C>
+cudaError_t setup_wave(int* occ) {
+  cudaError_t e = cudaFuncSetAttribute(nw_wave_kernel<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       static_cast<int>(C::kSmem));
+  if (e != cudaSuccess) return e;
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, nw_wave_kernel<C>, 32 * C::NW, C::kSmem);
 }
 
 std::mutex g_mu;
@@ -99,7 +122,14 @@ nw_status dev_info(int dev, DevInfo** out) {
     NW_CU((setup_kernel<CfgK2S>(&d.occ[0][1])));
     NW_CU((setup_kernel<CfgK4>(&d.occ[1][0])));
     NW_CU((setup_kernel<CfgK4S>(&d.occ[1][1])));
+    NW_CU((setup_wave<WCfgK2>(&d.wocc[0][0])));
+    NW_CU((setup_wave<WCfgK2S>(&d.wocc[0][1])));
+    NW_CU((setup_wave<WCfgK4>(&d.wocc[1][0])));
+    NW_CU((setup_wave<WCfgK4S>(&d.wocc[1][1])));
     for (auto& r : d.occ)
+      for (int o : r)
+        if (o < 1) return cuda_fail(cudaErrorInvalidConfiguration);
+    for (auto& r : d.wocc)
       for (int o : r)
         if (o < 1) return cuda_fail(cudaErrorInvalidConfiguration);
     d.init = true;
@@ -198,7 +228,8 @@ nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* 
   P.p = p;
   P.nbands = static_cast<int32_t>(nbands);
   P.ntasks = pairs * nbands;
-  const int NW = K == 2 ? CfgK2::NW : CfgK4::NW;
+  const bool wave = use_wave();
+  const int NW = wave ? (K == 2 ? WCfgK2::NW : WCfgK4::NW) : (K == 2 ? CfgK2::NW : CfgK4::NW);
   P.ngroups = (P.ntasks + NW - 1) / NW;
   P.xbuf = w->xbuf;
   P.epoch = ++w->epoch;
@@ -226,14 +257,23 @@ nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* 
     P.psb = psb;
     for (int i = 0; i < 32 * 32; ++i) P.subst[i] = subst32[i];
   }
-  const int occ = di->occ[K == 4][SEQ];
+  const int occ = wave ? di->wocc[K == 4][SEQ] : di->occ[K == 4][SEQ];
   int64_t grid = static_cast<int64_t>(occ) * di->sms;
   if (g_debug_grid > 0) grid = g_debug_grid;
   if (grid > P.ngroups) grid = P.ngroups;
   P.ticket_base = w->ticket_next;
   w->ticket_next += static_cast<unsigned long long>(P.ngroups + grid);  // every CTA draws one extra ticket
   const unsigned g = static_cast<unsigned>(grid);
-  if (K == 2 && !SEQ)
+  if (wave) {
+    if (K == 2 && !SEQ)
+      nw_wave_kernel<WCfgK2><<<g, 32 * WCfgK2::NW, WCfgK2::kSmem, st>>>(P);
+    else if (K == 2)
+      nw_wave_kernel<WCfgK2S><<<g, 32 * WCfgK2S::NW, WCfgK2S::kSmem, st>>>(P);
+    else if (!SEQ)
+      nw_wave_kernel<WCfgK4><<<g, 32 * WCfgK4::NW, WCfgK4::kSmem, st>>>(P);
+    else
+      nw_wave_kernel<WCfgK4S><<<g, 32 * WCfgK4S::NW, WCfgK4S::kSmem, st>>>(P);
+  } else if (K == 2 && !SEQ)
     nw_strip_kernel<CfgK2><<<g, 64 * CfgK2::NW, CfgK2::kSmem, st>>>(P);
   else if (K == 2)
     nw_strip_kernel<CfgK2S><<<g, 64 * CfgK2S::NW, CfgK2S::kSmem, st>>>(P);

@@ -1,3 +1,3 @@
 #!/bin/bash
 mkdir -p gpurun_out
-./scripts/ubench | tee gpurun_out/ubench.txt
+(./scripts/ubench; ./scripts/ubench_step) 2>&1 | tee gpurun_out/ubench.txt
