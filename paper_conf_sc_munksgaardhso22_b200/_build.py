@@ -18,7 +18,7 @@ SOURCES = ["nw_lib.cu"]
 DEPS = ["nw_lib.cu", "nw_strip.cuh", "nw_wave.cuh", "nw_diag.cuh", "nw_ptx.cuh"]
 
 NVCC_FLAGS = [
-    "-O3", "-std=c++17", "-lineinfo",
+    "-O3", "-std=c++20", "-lineinfo",
     "-gencode", "arch=compute_100a,code=sm_100a",
     "-Xcompiler", "-fPIC", "-shared", "--cudart", "static",
     "-Xptxas", "-v",

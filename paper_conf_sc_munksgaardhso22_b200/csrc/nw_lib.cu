@@ -14,7 +14,6 @@
 
 #include "nw.h"
 #include "nw_diag.cuh"
-#include "nw_strip.cuh"
 #include "nw_wave.cuh"
 
 using namespace nwb200;
@@ -36,12 +35,15 @@ nw_status cuda_fail(cudaError_t e) {
 
 constexpr int64_t kMaxN = (int64_t{1} << 30) - 64;
 
+// tile -> K (columns per lane) of the wavefront kernel: band width W = 32 K.  The paper's b x b
+// tiles (16/32/64) are narrower than one warp's band; they map to the W = 128 kernel.
 int tile_to_k(int32_t tile) {
   switch (tile) {
-    case 0: return 2;
+    case 0:
+    case 256: return 8;
     case 16:
     case 32:
-    case 64: return 2;
+    case 64:
     case 128: return 4;
     default: return 0;
   }
@@ -64,40 +66,19 @@ nw_status check_range(int64_t n, int32_t p) {
   return NW_OK;
 }
 
-// Kernel instances: K columns per lane, NW warps (bands) per CTA, CH-row staging chunks,
-// LOOK chunks of ref prefetch (DESIGN.md §4.3 sizes the rings).
-using CfgK2 = StripCfg<2, false, 4, 8, 64, 48>;
-using CfgK2S = StripCfg<2, true, 4, 8, 64, 48>;
-using CfgK4 = StripCfg<4, false, 2, 16, 96, 64>;
-using CfgK4S = StripCfg<4, true, 2, 16, 96, 64>;
+// Kernel instances: K columns per lane, SEQ (ref generated from the sequences), NW warps
+// (bands) per CTA (DESIGN.md §4.3 sizes the rings).
 // v5 self-staging wavefront kernels (nw_wave.cuh)
-using WCfgK2 = WaveCfg<2, false, 4>;
-using WCfgK2S = WaveCfg<2, true, 4>;
-using WCfgK4 = WaveCfg<4, false, 2>;
-using WCfgK4S = WaveCfg<4, true, 2>;
-
-bool use_wave() {
-  static const bool v = [] {
-    const char* e = std::getenv("NW_KERNEL");
-    return !(e && e[0] == 's');  // NW_KERNEL=strip selects the v4 kernel (A/B only)
-  }();
-  return v;
-}
+using WCfg8 = WaveCfg<8, false, 1>;   // tile 0 / 256: W = 256, one band per CTA
+using WCfg8S = WaveCfg<8, true, 1>;
+using WCfg4 = WaveCfg<4, false, 2>;   // tile 16 .. 128: W = 128, two bands per CTA
+using WCfg4S = WaveCfg<4, true, 2>;
 
 struct DevInfo {
   bool init = false;
   int sms = 0;
-  int occ[2][2] = {{0, 0}, {0, 0}};  // [K==4][SEQ]
-  int wocc[2][2] = {{0, 0}, {0, 0}};
+  int wocc[2][2] = {{0, 0}, {0, 0}};  // resident CTAs per SM [K==4][SEQ]
 };
-
-template <class C>
-cudaError_t setup_kernel(int* occ) {
-  cudaError_t e = cudaFuncSetAttribute(nw_strip_kernel<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       static_cast<int>(C::kSmem));
-  if (e != cudaSuccess) return e;
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, nw_strip_kernel<C>, 64 * C::NW, C::kSmem);
-}
 
 template <class C>
 cudaError_t setup_wave(int* occ) {
@@ -118,17 +99,10 @@ nw_status dev_info(int dev, DevInfo** out) {
   DevInfo& d = g_dev[dev];
   if (!d.init) {
     NW_CU(cudaDeviceGetAttribute(&d.sms, cudaDevAttrMultiProcessorCount, dev));
-    NW_CU((setup_kernel<CfgK2>(&d.occ[0][0])));
-    NW_CU((setup_kernel<CfgK2S>(&d.occ[0][1])));
-    NW_CU((setup_kernel<CfgK4>(&d.occ[1][0])));
-    NW_CU((setup_kernel<CfgK4S>(&d.occ[1][1])));
-    NW_CU((setup_wave<WCfgK2>(&d.wocc[0][0])));
-    NW_CU((setup_wave<WCfgK2S>(&d.wocc[0][1])));
-    NW_CU((setup_wave<WCfgK4>(&d.wocc[1][0])));
-    NW_CU((setup_wave<WCfgK4S>(&d.wocc[1][1])));
-    for (auto& r : d.occ)
-      for (int o : r)
-        if (o < 1) return cuda_fail(cudaErrorInvalidConfiguration);
+    NW_CU((setup_wave<WCfg8>(&d.wocc[0][0])));
+    NW_CU((setup_wave<WCfg8S>(&d.wocc[0][1])));
+    NW_CU((setup_wave<WCfg4>(&d.wocc[1][0])));
+    NW_CU((setup_wave<WCfg4S>(&d.wocc[1][1])));
     for (auto& r : d.wocc)
       for (int o : r)
         if (o < 1) return cuda_fail(cudaErrorInvalidConfiguration);
@@ -228,8 +202,7 @@ nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* 
   P.p = p;
   P.nbands = static_cast<int32_t>(nbands);
   P.ntasks = pairs * nbands;
-  const bool wave = use_wave();
-  const int NW = wave ? (K == 2 ? WCfgK2::NW : WCfgK4::NW) : (K == 2 ? CfgK2::NW : CfgK4::NW);
+  const int NW = K == 8 ? WCfg8::NW : WCfg4::NW;
   P.ngroups = (P.ntasks + NW - 1) / NW;
   P.xbuf = w->xbuf;
   P.epoch = ++w->epoch;
@@ -257,30 +230,21 @@ nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* 
     P.psb = psb;
     for (int i = 0; i < 32 * 32; ++i) P.subst[i] = subst32[i];
   }
-  const int occ = wave ? di->wocc[K == 4][SEQ] : di->occ[K == 4][SEQ];
+  const int occ = di->wocc[K == 4][SEQ];
   int64_t grid = static_cast<int64_t>(occ) * di->sms;
   if (g_debug_grid > 0) grid = g_debug_grid;
   if (grid > P.ngroups) grid = P.ngroups;
   P.ticket_base = w->ticket_next;
   w->ticket_next += static_cast<unsigned long long>(P.ngroups + grid);  // every CTA draws one extra ticket
   const unsigned g = static_cast<unsigned>(grid);
-  if (wave) {
-    if (K == 2 && !SEQ)
-      nw_wave_kernel<WCfgK2><<<g, 32 * WCfgK2::NW, WCfgK2::kSmem, st>>>(P);
-    else if (K == 2)
-      nw_wave_kernel<WCfgK2S><<<g, 32 * WCfgK2S::NW, WCfgK2S::kSmem, st>>>(P);
-    else if (!SEQ)
-      nw_wave_kernel<WCfgK4><<<g, 32 * WCfgK4::NW, WCfgK4::kSmem, st>>>(P);
-    else
-      nw_wave_kernel<WCfgK4S><<<g, 32 * WCfgK4S::NW, WCfgK4S::kSmem, st>>>(P);
-  } else if (K == 2 && !SEQ)
-    nw_strip_kernel<CfgK2><<<g, 64 * CfgK2::NW, CfgK2::kSmem, st>>>(P);
-  else if (K == 2)
-    nw_strip_kernel<CfgK2S><<<g, 64 * CfgK2S::NW, CfgK2S::kSmem, st>>>(P);
+  if (K == 8 && !SEQ)
+    nw_wave_kernel<WCfg8><<<g, 32 * WCfg8::NW, WCfg8::kSmem, st>>>(P);
+  else if (K == 8)
+    nw_wave_kernel<WCfg8S><<<g, 32 * WCfg8S::NW, WCfg8S::kSmem, st>>>(P);
   else if (!SEQ)
-    nw_strip_kernel<CfgK4><<<g, 64 * CfgK4::NW, CfgK4::kSmem, st>>>(P);
+    nw_wave_kernel<WCfg4><<<g, 32 * WCfg4::NW, WCfg4::kSmem, st>>>(P);
   else
-    nw_strip_kernel<CfgK4S><<<g, 64 * CfgK4S::NW, CfgK4S::kSmem, st>>>(P);
+    nw_wave_kernel<WCfg4S><<<g, 32 * WCfg4S::NW, WCfg4S::kSmem, st>>>(P);
   NW_CU(cudaGetLastError());
   return NW_OK;
 }
@@ -526,14 +490,14 @@ nw_status nw_kernel_info(int32_t tile, int32_t device, int64_t* smem_bytes, int3
                          int32_t* num_sms) {
   const int K = tile_to_k(tile);
   if (!K) return NW_EINVAL;
-  if (smem_bytes) *smem_bytes = static_cast<int64_t>(K == 2 ? CfgK2::kSmem : CfgK4::kSmem);
+  if (smem_bytes) *smem_bytes = static_cast<int64_t>(K == 8 ? WCfg8::kSmem : WCfg4::kSmem);
   if (!ctas_per_sm && !num_sms) return NW_OK;
   NW_CU(cudaSetDevice(device));
   std::lock_guard<std::mutex> lk(g_mu);
   DevInfo* di = nullptr;
   nw_status s = dev_info(device, &di);
   if (s != NW_OK) return s;
-  if (ctas_per_sm) *ctas_per_sm = di->occ[K == 4][0];
+  if (ctas_per_sm) *ctas_per_sm = di->wocc[K == 4][0];
   if (num_sms) *num_sms = di->sms;
   return NW_OK;
 }
