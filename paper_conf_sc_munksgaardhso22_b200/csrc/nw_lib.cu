@@ -85,7 +85,7 @@ cudaError_t setup_wave(int* occ) {
   cudaError_t e = cudaFuncSetAttribute(nw_wave_kernel<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        static_cast<int>(C::kSmem));
   if (e != cudaSuccess) return e;
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, nw_wave_kernel<C>, 32 * C::NW, C::kSmem);
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, nw_wave_kernel<C>, 64 * C::NW, C::kSmem);
 }
 
 std::mutex g_mu;
@@ -238,13 +238,13 @@ nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* 
   w->ticket_next += static_cast<unsigned long long>(P.ngroups + grid);  // every CTA draws one extra ticket
   const unsigned g = static_cast<unsigned>(grid);
   if (K == 8 && !SEQ)
-    nw_wave_kernel<WCfg8><<<g, 32 * WCfg8::NW, WCfg8::kSmem, st>>>(P);
+    nw_wave_kernel<WCfg8><<<g, 64 * WCfg8::NW, WCfg8::kSmem, st>>>(P);
   else if (K == 8)
-    nw_wave_kernel<WCfg8S><<<g, 32 * WCfg8S::NW, WCfg8S::kSmem, st>>>(P);
+    nw_wave_kernel<WCfg8S><<<g, 64 * WCfg8S::NW, WCfg8S::kSmem, st>>>(P);
   else if (!SEQ)
-    nw_wave_kernel<WCfg4><<<g, 32 * WCfg4::NW, WCfg4::kSmem, st>>>(P);
+    nw_wave_kernel<WCfg4><<<g, 64 * WCfg4::NW, WCfg4::kSmem, st>>>(P);
   else
-    nw_wave_kernel<WCfg4S><<<g, 32 * WCfg4S::NW, WCfg4S::kSmem, st>>>(P);
+    nw_wave_kernel<WCfg4S><<<g, 64 * WCfg4S::NW, WCfg4S::kSmem, st>>>(P);
   NW_CU(cudaGetLastError());
   return NW_OK;
 }

@@ -13,20 +13,23 @@
 //     each cell is two DPX VIADDMNMX (max-plus prefix form).
 //   * A CTA of NW warps claims NW consecutive bands through one atomic ticket (wavefront order;
 //     band k waits only on band k-1, so no deadlock without co-residency).
-//   * The kernel is issue-bound with one warp per SM sub-partition (measured: SHFL 24 cycles,
-//     DPX 4.75, LDS 29; scripts/ubench*.cu; ncu: "wait" + "selected" dominate), so the design
-//     minimises instructions per cell: wide bands (K = 8: 256 cells per step) and row-ALIGNED
-//     shared rings, so a lane's K ref values are K/4 LDS.128 and its K results K/4 STS.128.
-//   * The warp stages its own memory traffic, one row per step, interleaved with the sweep:
-//       - ref row s+LA: K 4-byte cp.async per lane (word 32i+t of the row segment -> ring word
-//         32i+t: the copy realigns the row whatever its 16-byte phase, which the Rodinia pitch
-//         n+1 changes from row to row), row s+PF prefetched into L2;
-//       - score row s-SD: K LDS.32 per lane, stored one step later with K coalesced STG.32.
+//   * The sweep is latency/issue bound with one warp per SM sub-partition (measured: SHFL 24
+//     cycles, DPX 4.75, LDS 29; scripts/ubench*.cu; ncu: "wait" + "selected" dominate), so the
+//     compute warp does nothing but the recurrence: wide bands (K = 8: 256 cells per step),
+//     row-ALIGNED shared rings (a lane's K ref values are K/4 LDS.128, its K results K/4
+//     STS.128), and a paired STAGING warp (another sub-partition) moves the memory traffic:
+//       - ref rows: K 4-byte cp.async per lane and row (word 32i+t of the row segment -> ring
+//         word 32i+t: the copy realigns the row whatever its 16-byte phase, which the Rodinia
+//         pitch n+1 changes from row to row), 8-row chunks, plus an L2 prefetch further ahead;
+//       - score rows: K LDS.32 + K coalesced STG.32 per lane and row.
 //     Ring row x of row r is (r-1) & 63; the row stride RS = W + 4*delta words shifts the
 //     16-byte bank group by delta per row, which makes the skewed LDS/STS.128 of the 32 lanes
 //     (32 different rows) conflict free (K=8: delta=1, K=4: delta=2).
-//   * Events every CH = 8 steps: cp.async commit / wait, border-block check, back-pressure,
-//     __syncwarp (ring writes of other lanes visible).  No other synchronisation inside a band.
+//     The two warps synchronise through two 64-bit progress words in shared memory (release /
+//     acquire, polled only when the cached value is insufficient): compute -> staging {ref rows
+//     consumed, score rows complete}, staging -> compute {ref rows landed, score rows stored}.
+//   * Compute-warp events every CH = 8 steps: progress words, border-block check (+ its cp.async
+//     commit / wait), back-pressure, __syncwarp.  No other synchronisation inside a band.
 //   * Band handoff (the paper's Fig. 9 ordering W ∩ R = ∅): the lane holding the band's last
 //     column publishes every row as a 64-bit entry {value, tag} (flag fused with the value):
 //       - to warp w+1 of the CTA: a 256-entry shared ring (tag = gen << 30 | row), back-pressure
@@ -55,26 +58,21 @@ struct WaveCfg {
   static constexpr int DELTA = K == 4 ? 2 : 1;  // 16-byte bank-group shift per ring row
   static constexpr int RS = W + 4 * DELTA;      // ring row stride (words)
   static constexpr int R = 64;                  // ring rows (ref and score rings)
-  static constexpr int LA = 26;                 // ref row s+LA issued at step s
-  static constexpr int SD = 40;                 // score row s-SD loaded at step s, stored at s+1
-  static constexpr int PF = LA + 64;            // L2 prefetch distance (rows)
+  static constexpr int PFC = 12;                // L2 prefetch distance (chunks of CH rows) of the staging warp
   static constexpr int BR = 256;                // shared border ring entries
   static constexpr int NL = (4 * W + 127) / 128 + 1;  // 128-byte lines touched by one row segment
   static constexpr int REF_WORDS = SEQ ? 0 : R * RS;
   static constexpr int PROF_WORDS = SEQ ? 32 * 32 * (K / 4) : 0;
   static constexpr int BPRE_BYTES = 4 * 8 * (CH + 2);  // border prefetch ring: 4 blocks x (CH+2) entries
-  static constexpr size_t kWarpSmem = 4ull * (REF_WORDS + R * RS + PROF_WORDS) + BPRE_BYTES;
+  static constexpr int HDR_BYTES = 128;                // progress words: [0] compute -> staging, [8] staging -> compute
+  static constexpr size_t kWarpSmem = HDR_BYTES + 4ull * (REF_WORDS + R * RS + PROF_WORDS) + BPRE_BYTES;
   static constexpr size_t kCtaHdr = 128 + static_cast<size_t>(NW - 1) * BR * 8;
   static constexpr size_t kSmem = kCtaHdr + NW * kWarpSmem;
   static_assert(K == 4 || K == 8, "K/4 LDS.128 per step");
   static_assert((RS * 4 / 16) % 8 == DELTA, "bank-group shift");
   static_assert(kWarpSmem % 16 == 0 && kCtaHdr % 16 == 0, "16-byte aligned rings");
   static_assert(NL <= 32 && NW <= 8, "geometry");
-  // LA: the wait at event Q completes block Q-3's copies (rows <= 8Q-17+LA), block Q reads rows
-  // <= 8Q+9; ring reuse: row r+R is issued at step r+R-LA, after an event that follows the last
-  // read of row r (step r+29).  SD: row r is complete after step r+30 and its slot is rewritten
-  // from step r+R-1 on, each side separated by an event.
-  static_assert(LA >= 26 && R - LA >= 30 + 1 && SD >= 30 + CH && SD + 1 <= R - 1 - CH, "staging distances");
+  static_assert(R % CH == 0 && (R & (R - 1)) == 0, "ring of whole chunks, power of two");
 };
 
 // ---- inline PTX helpers (immediate offsets keep the per-step staging at one instruction per copy)
@@ -133,36 +131,181 @@ __device__ __forceinline__ void st_entry_smem_p(bool pred, uint32_t a, uint32_t 
                : "memory");
 }
 
-// One band (task) swept by one warp.  RAGGED: the band is narrower than W (the last band of a
-// pair); its staging copies are predicated per word (full bands need no per-word predicate).
+// Shared per-band geometry of the compute and staging warps.
+template <class C>
+struct BandGeo {
+  int n, p, band, c0, ws;
+  bool last_band;
+  long long pair;
+  int32_t* S;
+  const int32_t* Rf;
+  uint32_t hdr, refR, scR, prof, bpre;  // shared addresses of the band's regions
+  __device__ __forceinline__ BandGeo(const StripParams& P, long long task, unsigned char* wsm) {
+    n = static_cast<int>(P.n);
+    p = P.p;
+    pair = task / P.nbands;
+    band = static_cast<int>(task - pair * P.nbands);
+    last_band = band == P.nbands - 1;
+    c0 = band_c0(band, C::W);
+    ws = band_ws(P.width, band, C::W);
+    S = P.score + pair * P.pss;
+    Rf = C::SEQ ? nullptr : P.ref + pair * P.psr;
+    hdr = smem_u32(wsm);
+    refR = hdr + C::HDR_BYTES;
+    scR = refR + 4u * C::REF_WORDS;
+    prof = scR + 4u * C::R * C::RS;
+    bpre = prof + 4u * C::PROF_WORDS;
+  }
+};
+
+// progress-word accessors (all lanes load: the value is uniform; lane 0 stores after __syncwarp)
+__device__ __forceinline__ void prog_publish(uint32_t a, int lo, int hi) {
+  __syncwarp();  // every lane's prior shared-memory accesses happen before lane 0's release
+  if ((threadIdx.x & 31) == 0) st_release_cta_v2(a, static_cast<uint32_t>(lo), static_cast<uint32_t>(hi));
+}
+__device__ __forceinline__ void prog_read(uint32_t a, int& lo, int& hi) {
+  const uint64_t v = ld_acquire_cta(a);
+  lo = static_cast<int>(static_cast<uint32_t>(v));
+  hi = static_cast<int>(static_cast<uint32_t>(v >> 32));
+}
+
+// The staging warp of a band: ref rows in (8-row chunks of 4-byte cp.async, paced by the ring
+// space the compute warp has released), score rows out (LDS.32 + coalesced STG.32 once the compute
+// warp has completed them), L2 prefetch ahead of the ref stream.
+template <class C, bool RAGGED>
+__device__ __forceinline__ void wave_stage(const StripParams& P, const long long task, const int t, unsigned char* const wsm) {
+  constexpr int K = C::K, CH = C::CH, R = C::R;
+  constexpr uint32_t RS4 = 4u * C::RS;
+  constexpr bool SEQ = C::SEQ;
+  const BandGeo<C> g(P, task, wsm);
+  const int n = g.n;
+  const int nch = (n + CH - 1) / CH;
+  const uint32_t from_c = g.hdr, to_c = g.hdr + 8;
+  uint32_t wmask = 0;  // RAGGED: bit i = word 32i+t of the row segment exists
+#pragma unroll
+  for (int i = 0; i < K; ++i) wmask |= static_cast<uint32_t>(32 * i + t < g.ws) << i;
+  const uint64_t ldr4 = 4ull * static_cast<uint64_t>(P.ldr), lds4 = 4ull * static_cast<uint64_t>(P.lds);
+  const uint64_t gR0 = SEQ ? 0ull : reinterpret_cast<uint64_t>(g.Rf + g.c0 + t);  // (row 0, word t) of the ref segment
+  const uint64_t gS0 = reinterpret_cast<uint64_t>(g.S + g.c0 + t);
+  const unsigned long long spin = P.spin_limit_ns;
+  auto wait_for = [&](int& cache_lo, int& cache_hi, bool want_lo, int need) {
+    // cached progress of the compute warp: lo = ref rows consumed, hi = score rows complete
+    int v = want_lo ? cache_lo : cache_hi;
+    if (v >= need) return;
+    const uint64_t tw = globaltimer_ns();
+    unsigned spins = 0;
+    for (;;) {
+      prog_read(from_c, cache_lo, cache_hi);
+      v = want_lo ? cache_lo : cache_hi;
+      if (v >= need) return;
+      if ((++spins & 255u) == 0 && globaltimer_ns() - tw > spin) watchdog_trap(P.err);
+    }
+  };
+  int consumed = 0, complete = 0;  // cached compute-warp progress
+  int landed = 0, stored = 0;      // published to the compute warp
+  // chunk k of ref: rows CH*k+1 .. CH*k+CH (row i of the chunk: K copies per lane)
+  auto issue_chunk = [&](int k) {
+    if constexpr (!SEQ) {
+#pragma unroll
+      for (int i = 0; i < CH; ++i) {
+        const int ri = CH * k + 1 + i;
+        const uint64_t gsrc = gR0 + static_cast<uint64_t>(static_cast<long long>(ri)) * ldr4;
+        const uint32_t d = g.refR + static_cast<uint32_t>((ri - 1) & (R - 1)) * RS4 + 4u * t;
+        if (ri <= n) {
+          if constexpr (!RAGGED) {
+            [&]<int... I>(std::integer_sequence<int, I...>) { (cp_async4_imm<128 * I>(d, gsrc), ...); }(std::make_integer_sequence<int, K>{});
+          } else {
+            [&]<int... I>(std::integer_sequence<int, I...>) {
+              (cp_async4_imm_p<128 * I>((wmask >> I) & 1u, d, gsrc), ...);
+            }(std::make_integer_sequence<int, K>{});
+          }
+        }
+      }
+    }
+  };
+  auto prefetch_chunk = [&](int k) {
+    if constexpr (!SEQ) {
+      // CH rows x NL lines, lane t handles lines t, t+32, ...
+#pragma unroll
+      for (int f = t; f < CH * C::NL; f += 32) {
+        const int i = f / C::NL, ln = f - (f / C::NL) * C::NL;
+        const int rp = CH * k + 1 + i;
+        const uint64_t ga = (reinterpret_cast<uint64_t>(g.Rf + g.c0) + static_cast<uint64_t>(static_cast<long long>(rp)) * ldr4) & ~127ull;
+        prefetch_l2_p(rp <= n, reinterpret_cast<const void*>(ga + 128u * ln));
+      }
+    }
+  };
+  auto store_chunk = [&](int k) {
+    int v[CH][K];
+#pragma unroll
+    for (int i = 0; i < CH; ++i) {
+      const int ro = CH * k + 1 + i;
+      const uint32_t a = g.scR + static_cast<uint32_t>((ro - 1) & (R - 1)) * RS4 + 4u * t;
+      [&]<int... I>(std::integer_sequence<int, I...>) { ((v[i][I] = lds32_imm<128 * I>(a)), ...); }(std::make_integer_sequence<int, K>{});
+    }
+#pragma unroll
+    for (int i = 0; i < CH; ++i) {
+      const int ro = CH * k + 1 + i;
+      const uint64_t ga = gS0 + static_cast<uint64_t>(static_cast<long long>(ro)) * lds4;
+      if constexpr (!RAGGED) {
+        [&]<int... I>(std::integer_sequence<int, I...>) { (stg32_imm_p<128 * I>(ro <= n, ga, v[i][I]), ...); }(std::make_integer_sequence<int, K>{});
+      } else {
+        [&]<int... I>(std::integer_sequence<int, I...>) {
+          (stg32_imm_p<128 * I>(ro <= n && ((wmask >> I) & 1u), ga, v[i][I]), ...);
+        }(std::make_integer_sequence<int, K>{});
+      }
+    }
+  };
+
+  // Iteration k: (1) publish the ref chunks landed (<= k-2) and score chunks stored (<= k-1-SK),
+  // (2) ref chunk k once rows <= CH*k+CH-R are consumed (ring space), (3) score chunk k-SK once
+  // complete.  The compute warp, at event Q, has consumed rows <= CH*Q-30, completed rows
+  // <= CH*Q-31 and needs ref rows <= CH*Q+9 landed and score rows <= CH*Q+CH-R stored: with
+  // R = 64 and SK = 9 every wait below is satisfiable (no deadlock), and ref chunk Q+1 is issued
+  // about two events before the compute warp needs it.
+  constexpr int SK = 9;
+  for (int k = 0; k < nch + SK; ++k) {
+    cp_async_wait<1>();  // chunks <= k-2 landed (this lane's copies)
+    const int nl = SEQ ? n : min(n, max(0, CH * (k - 1)));
+    const int ns = min(n, max(0, CH * (k - SK)));
+    if (nl > landed || ns > stored) {
+      landed = max(landed, nl);
+      stored = max(stored, ns);
+      prog_publish(to_c, landed, stored);  // __syncwarp: every lane's copies landed
+    }
+    if (!SEQ && k < nch) {
+      wait_for(consumed, complete, true, CH * k + CH - R);
+      issue_chunk(k);
+      if (k + C::PFC < nch) prefetch_chunk(k + C::PFC);
+    }
+    cp_async_commit();
+    const int js = k - SK;
+    if (js >= 0 && js < nch) {
+      wait_for(consumed, complete, false, min(n, CH * js + CH));
+      store_chunk(js);
+    }
+  }
+  prog_publish(to_c, n, n);
+}
+
+// The compute warp of a band: the wavefront sweep (no staging instructions in the step).
 template <class C, bool RAGGED>
 __device__ __forceinline__ void wave_band(const StripParams& P, const long long task, const int w, const int t,
                                           unsigned char* const smem, unsigned char* const wsm, const uint32_t gen,
                                           const int sink) {
-  constexpr int K = C::K, RS = C::RS, CH = C::CH, R = C::R;
-  constexpr uint32_t RS4 = 4u * RS;
+  constexpr int K = C::K, CH = C::CH, R = C::R;
+  constexpr uint32_t RS4 = 4u * C::RS;
   constexpr bool SEQ = C::SEQ;
   constexpr unsigned FULL = 0xffffffffu;
   const bool tracing = P.trace != nullptr;
   const unsigned long long t_task0 = tracing ? globaltimer_ns() : 0ull;
   long long spin_cyc = 0, ev_cyc = 0, bp_cyc = 0, wait_cyc = 0;
 
-  const int n = static_cast<int>(P.n);
-  const int p = P.p;
-  const long long pair = task / P.nbands;
-  const int band = static_cast<int>(task - pair * P.nbands);
-  const bool last_band = band == P.nbands - 1;
-  const int c0 = band_c0(band, C::W);
-  const int ws = band_ws(P.width, band, C::W);
-  int32_t* const S = P.score + pair * P.pss;
-  const int32_t* const Rf = SEQ ? nullptr : P.ref + pair * P.psr;
+  const BandGeo<C> g(P, task, wsm);
+  const int n = g.n, p = g.p, band = g.band, c0 = g.c0, ws = g.ws;
+  const long long pair = g.pair;
   const long long lds = P.lds;
-
-  // ---- shared layout of this warp
-  const uint32_t refR = opaque(smem_u32(wsm));
-  const uint32_t scR = opaque(smem_u32(wsm) + 4u * C::REF_WORDS);
-  uint32_t* const prof = reinterpret_cast<uint32_t*>(wsm + 4 * (C::REF_WORDS + R * RS));
-  const uint32_t bpre = smem_u32(wsm) + 4u * (C::REF_WORDS + R * RS + C::PROF_WORDS);
+  const uint32_t to_s = g.hdr, from_s = g.hdr + 8;
   const uint32_t s_prog = smem_u32(smem + 8);     // [4w]: rows consumed by warp w (shared source)
   const uint32_t s_bring = smem_u32(smem + 128);  // [w * BR * 8]: ring warp w -> w+1
 
@@ -187,14 +330,14 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
   const uint32_t bring_out = s_bring + w * C::BR * 8;
   const uint32_t prog_in = s_prog + 4 * w;         // written by this warp (consumer of w-1)
   const uint32_t prog_out = s_prog + 4 * (w + 1);  // read by this warp (producer for w+1)
-  const int32_t* const colp = S + (c0 - 1);        // plain left border column
+  const int32_t* const colp = g.S + (c0 - 1);      // plain left border column
   // ---- sink (right)
   uint64_t* lout = nullptr;
   uint32_t lout_tag = 0;
   const bool sink_smem = sink == kSinkSmem;
   bool sink_gpu = false, sink_sys = false;
   if (sink == kSinkGlobal) {
-    if (last_band) {
+    if (g.last_band) {
       lout = P.halo_out;
       lout_tag = P.halo_epoch;
       sink_sys = P.halo_out_sys != 0;
@@ -217,12 +360,13 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     if (src == kSrcSmem) return lds64_volatile(bring_in + 8u * (row & (C::BR - 1)));
     return static_cast<uint32_t>(__ldg(colp + static_cast<long long>(row) * lds));
   };
-  // Global / plain sources: block q is copied by cp.async three blocks ahead (it joins the
-  // commit group of that block, so the event's wait covers it) into slot q & 3 of a shared ring:
-  // rows CH*q .. CH*q+CH+1 (global: 16-byte pairs (2k, 2k+1) through L2 only, never via L1 since
-  // the entries are polled; plain: the 4-byte values of score column c0-1).
+  // Global / plain sources: block q is copied by cp.async three blocks ahead (one commit group
+  // per event, so the event's wait covers it) into slot q & 3 of a shared ring: rows
+  // CH*q .. CH*q+CH+1 (global: 16-byte pairs (2k, 2k+1) through L2 only, never via L1 since the
+  // entries are polled; plain: the 4-byte values of score column c0-1).  No register holds an
+  // in-flight load across an event (a register move of one stalls the warp for the latency).
   auto prefetch_block = [&](int q) {
-    const uint32_t slot = bpre + 8u * (CH + 2) * static_cast<uint32_t>(q & 3);
+    const uint32_t slot = g.bpre + 8u * (CH + 2) * static_cast<uint32_t>(q & 3);
     if (src == kSrcGlobal) {
       const int row = CH * q + 2 * t;
       cp_async16_cg_p(t <= CH / 2 && row <= n, slot + 16u * t, lin + row);
@@ -232,7 +376,7 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     }
   };
   auto read_block = [&](int q) -> uint64_t {
-    const uint32_t slot = bpre + 8u * (CH + 2) * static_cast<uint32_t>(q & 3);
+    const uint32_t slot = g.bpre + 8u * (CH + 2) * static_cast<uint32_t>(q & 3);
     return t < CH ? lds64_volatile(slot + 8u * (1 + t)) : 0ull;
   };
   auto block_ok = [&](uint64_t e, int q) -> bool {
@@ -248,76 +392,23 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     return __all_sync(FULL, ok) != 0;
   };
 
-  // ---- staging state: lane t moves words 32i+t (i < K) of each staged row
-  uint32_t wmask = 0;  // RAGGED: bit i = word 32i+t of the row segment exists
-#pragma unroll
-  for (int i = 0; i < K; ++i) wmask |= static_cast<uint32_t>(32 * i + t < ws) << i;
-  const uint64_t gR0 = SEQ ? 0ull : reinterpret_cast<uint64_t>(Rf + c0 + t);  // (row 0, word t) of the ref segment
-  const uint64_t gS0 = reinterpret_cast<uint64_t>(S + c0 + t);
-  const uint64_t ldr4 = 4ull * static_cast<uint64_t>(P.ldr), lds4 = 4ull * static_cast<uint64_t>(lds);
-  // one ref row -> ring
-  auto issue_ref = [&](int ri, bool ok) {
-    if constexpr (!SEQ) {
-      const uint64_t g = gR0 + static_cast<uint64_t>(static_cast<long long>(ri)) * ldr4;
-      const uint32_t d = refR + static_cast<uint32_t>((ri - 1) & (R - 1)) * RS4 + 4u * t;
-      if (ok) {
-        if constexpr (!RAGGED) {
-          [&]<int... I>(std::integer_sequence<int, I...>) { (cp_async4_imm<128 * I>(d, g), ...); }(std::make_integer_sequence<int, K>{});
-        } else {
-          [&]<int... I>(std::integer_sequence<int, I...>) {
-            (cp_async4_imm_p<128 * I>((wmask >> I) & 1u, d, g), ...);
-          }(std::make_integer_sequence<int, K>{});
-        }
-      }
-    }
-  };
-  auto prefetch_ref = [&](int rp) {
-    if constexpr (!SEQ) {
-      const uint64_t g = (reinterpret_cast<uint64_t>(Rf + c0) + static_cast<uint64_t>(static_cast<long long>(rp)) * ldr4) & ~127ull;
-      prefetch_l2_p(t < C::NL && rp >= 1 && rp <= n, reinterpret_cast<const void*>(g + 128u * t));
-    }
-  };
-  // score rows leave software-pipelined: LDS at step s (row s-SD), STG at step s+1
-  int sv[K];
-#pragma unroll
-  for (int i = 0; i < K; ++i) sv[i] = 0;
-  uint64_t sga = 0;
-  bool sgo = false;
-  auto store_step = [&](int ro) {
-    // the row loaded last step
-    if constexpr (!RAGGED) {
-      [&]<int... I>(std::integer_sequence<int, I...>) { (stg32_imm_p<128 * I>(sgo, sga, sv[I]), ...); }(std::make_integer_sequence<int, K>{});
-    } else {
-      [&]<int... I>(std::integer_sequence<int, I...>) {
-        (stg32_imm_p<128 * I>(sgo && ((wmask >> I) & 1u), sga, sv[I]), ...);
-      }(std::make_integer_sequence<int, K>{});
-    }
-    sgo = ro >= 1 && ro <= n;
-    sga = gS0 + static_cast<uint64_t>(static_cast<long long>(ro)) * lds4;
-    const uint32_t a = scR + static_cast<uint32_t>((ro - 1) & (R - 1)) * RS4 + 4u * t;
-    [&]<int... I>(std::integer_sequence<int, I...>) { ((sv[I] = lds32_imm<128 * I>(a)), ...); }(std::make_integer_sequence<int, K>{});
-  };
-
-  // ---- prologue: top border row, first border blocks, ref rows 1 .. LA-1
+  // ---- prologue: top border row, first border blocks
   int Pv[K];
 #pragma unroll
-  for (int m = 0; m < K; ++m) Pv[m] = (t * K + m < ws) ? __ldg(S + c0 + t * K + m) : 0;
-  int Lprev = (t * K < ws) ? __ldg(S + c0 + t * K - 1) : 0;  // diag input of the first row
-  uint64_t e1 = src == kSrcSmem ? load_block(0) : 0ull;      // shared source: the next block's entries
+  for (int m = 0; m < K; ++m) Pv[m] = (t * K + m < ws) ? __ldg(g.S + c0 + t * K + m) : 0;
+  int Lprev = (t * K < ws) ? __ldg(g.S + c0 + t * K - 1) : 0;  // diag input of the first row
+  uint64_t e1 = src == kSrcSmem ? load_block(0) : 0ull;        // shared source: the next block's entries
   if (src != kSrcSmem)
     for (int q = 0; q < 3; ++q) prefetch_block(q);
-  // three commit groups before event 0 (event Q's wait completes the group of block Q-3); the
-  // first holds the border blocks 0..2 and every ref row issued before step 0
-  for (int ri = 1; ri < C::LA; ++ri) issue_ref(ri, ri <= n);
+  cp_async_commit();  // three groups before event 0: event Q's wait completes block Q-3's group
   cp_async_commit();
   cp_async_commit();
-  cp_async_commit();
-  for (int rp = C::LA; rp < C::PF; rp += 2) prefetch_ref(rp);  // every other row: lines overlap
 
   // SEQ: per-band substitution profile prof[x][t] = pack_m subst[x][b[c0-1+tK+m]] (int8 x K)
   const uint8_t* const A = SEQ ? P.seq_a + pair * P.psa : nullptr;
   int a_cur = 0, a_nxt = 0;  // residues of this lane's current / next row (software pipeline)
   if constexpr (SEQ) {
+    uint32_t* const prof = reinterpret_cast<uint32_t*>(wsm + (g.prof - g.hdr));
     const uint8_t* const Bq = P.seq_b + pair * P.psb;
     int bj[K];
 #pragma unroll
@@ -335,19 +426,20 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     a_nxt = A[min(max(1 - t, 0), n - 1)] & 31;  // row 2-t
     __syncwarp();
   }
-  const uint32_t profA = smem_u32(prof) + 4u * (K / 4) * t;
+  const uint32_t profA = g.prof + 4u * (K / 4) * t;
 
   int negp[K];  // -(m+1) p
 #pragma unroll
   for (int m = 0; m < K; ++m) negp[m] = static_cast<int>(opaque(static_cast<uint32_t>(-(m + 1) * p)));
-  uint32_t tok = 0;  // produced after each event's wait, consumed by the ref loads
+  uint32_t tok = 0;  // produced after each event's acquire, consumed by the ref loads
   int rvn[K];        // ref of the lane's NEXT row (loaded one step ahead)
 #pragma unroll
   for (int m = 0; m < K; ++m) rvn[m] = 0;
-  int bp_cache = 0;  // last consumer progress read (back-pressure, shared sink)
+  int bp_cache = 0;            // last consumer progress read (back-pressure, shared sink)
+  int landed = 0, stored = 0;  // cached staging-warp progress
   uint64_t cur = 0ull;
   int vlast = Pv[K - 1];
-  const uint32_t laneR = refR + 16u * (K / 4) * t, laneS = scR + 16u * (K / 4) * t;
+  const uint32_t laneR = opaque(g.refR + 16u * (K / 4) * t), laneS = opaque(g.scR + 16u * (K / 4) * t);
   auto load_ref_row = [&](uint32_t a) {  // K/4 LDS.128 of this lane's K ref values
     const int4 u = lds128_tok<0>(a, tok);
     rvn[0] = u.x, rvn[1] = u.y, rvn[2] = u.z, rvn[3] = u.w;
@@ -357,15 +449,10 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     }
   };
 
-  // one wavefront step s = CH*Q + j; ALL = every lane's row is in 1..n and every staged row
-  // exists (no predicates)
+  // one wavefront step s = CH*Q + j; ALL = every lane's row is in 1..n (no predicates)
   auto step = [&](const int s, const int j, auto all_tag) {
     constexpr bool ALL = decltype(all_tag)::value;
     const int r = s + 1 - t;  // this lane's row
-    // ---- staging (independent of the recurrence: fills the issue slots it leaves idle)
-    issue_ref(s + C::LA, ALL || s + C::LA <= n);
-    if (j & 1) prefetch_ref(s + C::PF);
-    store_step(s - C::SD);
     // ---- ref of this step's row (loaded last step) and the next row's loads
     int rv[K];
     if constexpr (SEQ) {
@@ -385,8 +472,7 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     } else {
 #pragma unroll
       for (int m = 0; m < K; ++m) rv[m] = rvn[m];
-      const uint32_t an = laneR + static_cast<uint32_t>(r & (R - 1)) * RS4;  // ring row of row r+1
-      load_ref_row(an);
+      load_ref_row(laneR + static_cast<uint32_t>(r & (R - 1)) * RS4);  // ring row of row r+1
     }
     // ---- left value: lane t-1's last column of this row, lane 0: the border entry
     const int bval = __shfl_sync(FULL, static_cast<int>(static_cast<uint32_t>(cur)), j);
@@ -424,16 +510,32 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     vlast = Pv[K - 1];
   };
 
-  const int nsteps = n + 31;                  // compute steps 0 .. n+30
-  const int nblk = (n + C::SD + 1) / CH + 1;  // the last score row is stored at step n+SD+1
+  const int nsteps = n + 31;  // compute steps 0 .. n+30
+  const int nblk = (nsteps + CH - 1) / CH;
   for (int Q = 0; Q < nblk; ++Q) {
     const int sig0 = Q * CH;
     const long long c_ev0 = tracing ? clock64() : 0;
-    // ---- event Q
-    cp_async_commit();   // copies issued during block Q-1 (ref rows, border block Q+2)
-    cp_async_wait<2>();  // block Q-3's copies landed: ref rows <= CH*Q-17+LA, border block Q
-    if (tracing) wait_cyc += clock64() - c_ev0;
-    __syncwarp();        // ring writes of every lane (cp.async landed, score STS) visible warp-wide
+    // ---- event Q.  To the staging warp: ref rows <= sig0-30 consumed (lane 31 read row sig0-30
+    // at step sig0-1), score rows <= sig0-31 complete (lane 31 wrote row sig0-31 at step sig0-1).
+    prog_publish(to_s, max(0, sig0 - 30), max(0, sig0 - 31));
+    {
+      // this block reads ref rows <= sig0+CH+1 and rewrites score slots of rows <= sig0+CH
+      const int need_l = SEQ ? 0 : min(n, sig0 + CH + 1), need_s = sig0 + CH - R;
+      if (landed < need_l || stored < need_s) {
+        const long long c0c = clock64();
+        const uint64_t tw = globaltimer_ns();
+        unsigned spins = 0;
+        for (;;) {
+          prog_read(from_s, landed, stored);
+          if (landed >= need_l && stored >= need_s) break;
+          if ((++spins & 255u) == 0 && globaltimer_ns() - tw > P.spin_limit_ns) watchdog_trap(P.err);
+        }
+        wait_cyc += clock64() - c0c;
+      }
+    }
+    cp_async_commit();   // the border copies issued at event Q-1 (block Q+2)
+    cp_async_wait<2>();  // block Q's border entries landed
+    __syncwarp();        // cp.async landed by lanes 0..CH-1 visible to the warp
     if (sig0 < nsteps) {
       if (src == kSrcSmem) {
         cur = e1;
@@ -467,14 +569,11 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     }
     asm volatile("mov.u32 %0, 0;" : "=r"(tok)::"memory");  // the block's ref loads stay below
     if constexpr (!SEQ) {
-      if (Q == 0) {  // the first row's ref values (row 1-t, ring row -t & (R-1))
-        const uint32_t a0 = laneR + static_cast<uint32_t>((-t) & (R - 1)) * RS4;
-        load_ref_row(a0);
-      }
+      if (Q == 0) load_ref_row(laneR + static_cast<uint32_t>((-t) & (R - 1)) * RS4);  // row 1-t
     }
     if (tracing) ev_cyc += clock64() - c_ev0;
     // ---- CH steps
-    if (sig0 >= 31 && sig0 + CH <= n - C::LA && sig0 >= C::SD + 1) {
+    if (sig0 >= 31 && sig0 + CH <= n) {
 #pragma unroll
       for (int j = 0; j < CH; ++j) step(sig0 + j, j, std::true_type{});
     } else {
@@ -482,6 +581,7 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
       for (int j = 0; j < CH; ++j) step(sig0 + j, j, std::false_type{});
     }
   }
+  prog_publish(to_s, n, n);  // every row consumed and complete
   if (tracing && t == 0 && task < P.trace_cap) {
     unsigned smid;
     asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
@@ -498,18 +598,24 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
 }
 
 template <class C>
-__global__ void __launch_bounds__(32 * C::NW, 1) nw_wave_kernel(const __grid_constant__ StripParams P) {
+__global__ void __launch_bounds__(64 * C::NW, 1) nw_wave_kernel(const __grid_constant__ StripParams P) {
   constexpr int NW = C::NW;
   extern __shared__ __align__(128) unsigned char smem[];
   const int t = threadIdx.x & 31;
-  const int w = threadIdx.x >> 5;
+  const int wa = threadIdx.x >> 5;  // 0..NW-1 compute warps, NW..2NW-1 staging warps
+  const bool staging = wa >= NW;
+  const int w = staging ? wa - NW : wa;  // the band slot this warp serves
   // CTA header: [0] group ticket, [8 + 4w] consumer progress of warp w, [128..] border rings
   unsigned long long* const s_group = reinterpret_cast<unsigned long long*>(smem);
   const uint32_t s_prog = smem_u32(smem + 8);
   unsigned char* const wsm = smem + C::kCtaHdr + w * C::kWarpSmem;
   // shared border rings start invalid (tag 0xFFFFFFFF never equals gen | row, row < 2^30)
-  for (int i = threadIdx.x; i < (NW - 1) * C::BR; i += 32 * NW) reinterpret_cast<unsigned long long*>(smem + 128)[i] = ~0ull;
+  for (int i = threadIdx.x; i < (NW - 1) * C::BR; i += 64 * NW) reinterpret_cast<unsigned long long*>(smem + 128)[i] = ~0ull;
   if (threadIdx.x < NW) sts32_volatile(s_prog + 4 * threadIdx.x, 0);
+  if (!staging && t == 0) {  // band progress words
+    st_release_cta_v2(smem_u32(wsm), 0u, 0u);
+    st_release_cta_v2(smem_u32(wsm) + 8, 0u, 0u);
+  }
   __syncthreads();
 
   int gcount = 0;  // groups processed by this CTA (generation of the shared border tags)
@@ -522,19 +628,32 @@ __global__ void __launch_bounds__(32 * C::NW, 1) nw_wave_kernel(const __grid_con
     const uint32_t gen = static_cast<uint32_t>(gcount & 3) << 30;
     if (task < P.ntasks) {
       const int band = static_cast<int>(task % P.nbands);
-      const bool last_band = band == P.nbands - 1;
-      int sink;
-      if (last_band)
-        sink = P.halo_out ? kSinkGlobal : kSinkNone;
-      else
-        sink = (w < NW - 1) ? kSinkSmem : kSinkGlobal;
-      if (band_ws(P.width, band, C::W) == C::W)
-        wave_band<C, false>(P, task, w, t, smem, wsm, gen, sink);
-      else
-        wave_band<C, true>(P, task, w, t, smem, wsm, gen, sink);
+      const bool full = band_ws(P.width, band, C::W) == C::W;
+      if (staging) {
+        if (full)
+          wave_stage<C, false>(P, task, t, wsm);
+        else
+          wave_stage<C, true>(P, task, t, wsm);
+      } else {
+        const bool last_band = band == P.nbands - 1;
+        int sink;
+        if (last_band)
+          sink = P.halo_out ? kSinkGlobal : kSinkNone;
+        else
+          sink = (w < NW - 1) ? kSinkSmem : kSinkGlobal;
+        if (full)
+          wave_band<C, false>(P, task, w, t, smem, wsm, gen, sink);
+        else
+          wave_band<C, true>(P, task, w, t, smem, wsm, gen, sink);
+      }
     }
-    __syncthreads();  // group end: every warp done (shared border rings / progress reusable)
+    __syncthreads();  // group end: every warp done (shared rings / progress words reusable)
     if (threadIdx.x < NW) sts32_volatile(s_prog + 4 * threadIdx.x, 0);
+    if (!staging && t == 0) {
+      st_release_cta_v2(smem_u32(wsm), 0u, 0u);
+      st_release_cta_v2(smem_u32(wsm) + 8, 0u, 0u);
+    }
+    __syncthreads();
     ++gcount;
   }
 }
