@@ -28,11 +28,12 @@
  *   - Device pointers are owned by the caller and must be 4-byte aligned.
  *   - `stream` is a cudaStream_t (NULL = legacy default stream).  Work is ENQUEUED and the
  *     call returns; results are visible after the caller synchronises the stream.
- *   - `tile` b in {0, 16, 32, 64, 128} selects the width W of the tile-column band one warp
- *     owns (W = 32K, K columns per lane): b in {0, 16, 32, 64} -> W = 64 (K = 2, the default;
- *     narrower b x b tiles are processed 64/b side by side, because conflict-free shared
- *     staging needs an even K), b = 128 -> W = 128 (K = 4).  A CTA of 4 (K=2) or 2 (K=4) warps
- *     owns that many consecutive bands.  The result does not depend on it (R8).
+ *   - `tile` b in {0, 16, 32, 64, 128, 256} selects the width W of the tile-column band one
+ *     warp owns (W = 32K, K columns per lane): b in {0, 16, 32, 64, 128} -> W = 128 (K = 4, the
+ *     default; narrower b x b tiles are processed 128/b side by side, because a lane's K ref
+ *     values are one 16-byte shared load), b = 256 -> W = 256 (K = 8).  A CTA owns 2 (K=4) or
+ *     1 (K=8) consecutive bands, each swept by a compute warp paired with a staging warp.  The
+ *     result does not depend on it (R8).
  *   - Any n >= 0 is accepted (ragged last band: n need not be a multiple of b).
  *   - Validation is synchronous and happens before anything is enqueued.  Range contract:
  *     0 <= penalty and 2*n*penalty + n*NW_REF_MAX < 2^31 (else NW_ERANGE), |ref| <= NW_REF_MAX

@@ -36,15 +36,16 @@ nw_status cuda_fail(cudaError_t e) {
 constexpr int64_t kMaxN = (int64_t{1} << 30) - 64;
 
 // tile -> K (columns per lane) of the wavefront kernel: band width W = 32 K.  The paper's b x b
-// tiles (16/32/64) are narrower than one warp's band; they map to the W = 128 kernel.
+// tiles (16/32/64) are narrower than one warp's band; they map to the W = 128 kernel (the
+// default, measured fastest at n = 32768); tile 256 selects the W = 256 kernel.
 int tile_to_k(int32_t tile) {
   switch (tile) {
     case 0:
-    case 256: return 8;
     case 16:
     case 32:
     case 64:
     case 128: return 4;
+    case 256: return 8;
     default: return 0;
   }
 }
@@ -69,9 +70,9 @@ nw_status check_range(int64_t n, int32_t p) {
 // Kernel instances: K columns per lane, SEQ (ref generated from the sequences), NW warps
 // (bands) per CTA (DESIGN.md §4.3 sizes the rings).
 // v5 self-staging wavefront kernels (nw_wave.cuh)
-using WCfg8 = WaveCfg<8, false, 1>;   // tile 0 / 256: W = 256, one band per CTA
+using WCfg8 = WaveCfg<8, false, 1>;   // tile 256: W = 256, one band per CTA
 using WCfg8S = WaveCfg<8, true, 1>;
-using WCfg4 = WaveCfg<4, false, 2>;   // tile 16 .. 128: W = 128, two bands per CTA
+using WCfg4 = WaveCfg<4, false, 2>;   // tile 0 / 16 .. 128: W = 128, two bands per CTA
 using WCfg4S = WaveCfg<4, true, 2>;
 
 struct DevInfo {

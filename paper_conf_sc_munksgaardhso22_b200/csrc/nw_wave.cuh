@@ -54,25 +54,28 @@ struct WaveCfg {
   static constexpr int K = K_, NW = NW_;
   static constexpr bool SEQ = SEQ_;
   static constexpr int W = 32 * K;
-  static constexpr int CH = 8;                  // event period (steps) = border block (rows)
+  static constexpr int CH = 8;                  // staging chunk (rows)
+  static constexpr int CE = 16;                 // compute-warp event period (steps) = border block (rows)
   static constexpr int DELTA = K == 4 ? 2 : 1;  // 16-byte bank-group shift per ring row
   static constexpr int RS = W + 4 * DELTA;      // ring row stride (words)
-  static constexpr int R = 64;                  // ring rows (ref and score rings)
+  static constexpr int RR = 128;                // ref ring rows (the staging warp's lookahead)
+  static constexpr int SR = 64;                 // score ring rows
   static constexpr int PFC = 12;                // L2 prefetch distance (chunks of CH rows) of the staging warp
   static constexpr int BR = 256;                // shared border ring entries
   static constexpr int NL = (4 * W + 127) / 128 + 1;  // 128-byte lines touched by one row segment
-  static constexpr int REF_WORDS = SEQ ? 0 : R * RS;
+  static constexpr int REF_WORDS = SEQ ? 0 : RR * RS;
   static constexpr int PROF_WORDS = SEQ ? 32 * 32 * (K / 4) : 0;
-  static constexpr int BPRE_BYTES = 4 * 8 * (CH + 2);  // border prefetch ring: 4 blocks x (CH+2) entries
+  static constexpr int BPRE_BYTES = 4 * 8 * (CE + 2);  // border prefetch ring: 4 blocks x (CE+2) entries
   static constexpr int HDR_BYTES = 128;                // progress words: [0] compute -> staging, [8] staging -> compute
-  static constexpr size_t kWarpSmem = HDR_BYTES + 4ull * (REF_WORDS + R * RS + PROF_WORDS) + BPRE_BYTES;
+  static constexpr size_t kWarpSmem = HDR_BYTES + 4ull * (REF_WORDS + SR * RS + PROF_WORDS) + BPRE_BYTES;
   static constexpr size_t kCtaHdr = 128 + static_cast<size_t>(NW - 1) * BR * 8;
   static constexpr size_t kSmem = kCtaHdr + NW * kWarpSmem;
   static_assert(K == 4 || K == 8, "K/4 LDS.128 per step");
   static_assert((RS * 4 / 16) % 8 == DELTA, "bank-group shift");
   static_assert(kWarpSmem % 16 == 0 && kCtaHdr % 16 == 0, "16-byte aligned rings");
   static_assert(NL <= 32 && NW <= 8, "geometry");
-  static_assert(R % CH == 0 && (R & (R - 1)) == 0, "ring of whole chunks, power of two");
+  static_assert(RR % CH == 0 && (RR & (RR - 1)) == 0 && SR % CH == 0 && (SR & (SR - 1)) == 0 && RR >= 64 && SR >= 64,
+                "rings of whole chunks, powers of two, large enough for the staging schedule");
 };
 
 // ---- inline PTX helpers (immediate offsets keep the per-step staging at one instruction per copy)
@@ -153,15 +156,20 @@ struct BandGeo {
     hdr = smem_u32(wsm);
     refR = hdr + C::HDR_BYTES;
     scR = refR + 4u * C::REF_WORDS;
-    prof = scR + 4u * C::R * C::RS;
+    prof = scR + 4u * C::SR * C::RS;
     bpre = prof + 4u * C::PROF_WORDS;
   }
 };
 
 // progress-word accessors (all lanes load: the value is uniform; lane 0 stores after __syncwarp)
-__device__ __forceinline__ void prog_publish(uint32_t a, int lo, int hi) {
+__device__ __forceinline__ void prog_publish(uint32_t a, int lo, int hi, bool relaxed = false) {
   __syncwarp();  // every lane's prior shared-memory accesses happen before lane 0's release
-  if ((threadIdx.x & 31) == 0) st_release_cta_v2(a, static_cast<uint32_t>(lo), static_cast<uint32_t>(hi));
+  if ((threadIdx.x & 31) == 0) {
+    if (relaxed)
+      asm volatile("{ .reg .b64 e; mov.b64 e, {%1, %2}; st.volatile.shared.b64 [%0], e; }" ::"r"(a), "r"(lo), "r"(hi) : "memory");
+    else
+      st_release_cta_v2(a, static_cast<uint32_t>(lo), static_cast<uint32_t>(hi));
+  }
 }
 __device__ __forceinline__ void prog_read(uint32_t a, int& lo, int& hi) {
   const uint64_t v = ld_acquire_cta(a);
@@ -174,7 +182,7 @@ __device__ __forceinline__ void prog_read(uint32_t a, int& lo, int& hi) {
 // warp has completed them), L2 prefetch ahead of the ref stream.
 template <class C, bool RAGGED>
 __device__ __forceinline__ void wave_stage(const StripParams& P, const long long task, const int t, unsigned char* const wsm) {
-  constexpr int K = C::K, CH = C::CH, R = C::R;
+  constexpr int K = C::K, CH = C::CH, RR = C::RR, SR = C::SR;
   constexpr uint32_t RS4 = 4u * C::RS;
   constexpr bool SEQ = C::SEQ;
   const BandGeo<C> g(P, task, wsm);
@@ -210,7 +218,7 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
       for (int i = 0; i < CH; ++i) {
         const int ri = CH * k + 1 + i;
         const uint64_t gsrc = gR0 + static_cast<uint64_t>(static_cast<long long>(ri)) * ldr4;
-        const uint32_t d = g.refR + static_cast<uint32_t>((ri - 1) & (R - 1)) * RS4 + 4u * t;
+        const uint32_t d = g.refR + static_cast<uint32_t>((ri - 1) & (RR - 1)) * RS4 + 4u * t;
         if (ri <= n) {
           if constexpr (!RAGGED) {
             [&]<int... I>(std::integer_sequence<int, I...>) { (cp_async4_imm<128 * I>(d, gsrc), ...); }(std::make_integer_sequence<int, K>{});
@@ -240,7 +248,7 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
 #pragma unroll
     for (int i = 0; i < CH; ++i) {
       const int ro = CH * k + 1 + i;
-      const uint32_t a = g.scR + static_cast<uint32_t>((ro - 1) & (R - 1)) * RS4 + 4u * t;
+      const uint32_t a = g.scR + static_cast<uint32_t>((ro - 1) & (SR - 1)) * RS4 + 4u * t;
       [&]<int... I>(std::integer_sequence<int, I...>) { ((v[i][I] = lds32_imm<128 * I>(a)), ...); }(std::make_integer_sequence<int, K>{});
     }
 #pragma unroll
@@ -257,49 +265,82 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
     }
   };
 
-  // Iteration k: (1) publish the ref chunks landed (<= k-2) and score chunks stored (<= k-1-SK),
-  // (2) ref chunk k once rows <= CH*k+CH-R are consumed (ring space), (3) score chunk k-SK once
-  // complete.  The compute warp, at event Q, has consumed rows <= CH*Q-30, completed rows
-  // <= CH*Q-31 and needs ref rows <= CH*Q+9 landed and score rows <= CH*Q+CH-R stored: with
-  // R = 64 and SK = 9 every wait below is satisfiable (no deadlock), and ref chunk Q+1 is issued
-  // about two events before the compute warp needs it.
-  constexpr int SK = 9;
-  for (int k = 0; k < nch + SK; ++k) {
-    cp_async_wait<1>();  // chunks <= k-2 landed (this lane's copies)
-    const int nl = SEQ ? n : min(n, max(0, CH * (k - 1)));
-    const int ns = min(n, max(0, CH * (k - SK)));
+  // Event loop (never blocks on one side while the other could progress): issue ref chunk kr
+  // once rows <= CH*kr+CH-RR are consumed (ring space), store score chunk ks once complete, and
+  // publish the ref chunks landed (all but the LAG most recent) and the score chunks stored.  The
+  // compute warp, at event Q (step CE*Q), has consumed ref rows <= CE*Q-30 and completed score
+  // rows <= CE*Q-31, and needs ref rows <= CE*Q+CE+1 landed and score rows <= CE*Q+CE-SR stored:
+  // with RR = 128 the ref stream runs about RR/2 rows ahead, so both waits are satisfiable
+  // (no deadlock) and normally already satisfied.
+  constexpr int LAG = 3;
+  int kr = SEQ ? nch : 0, ks = 0;
+  const uint64_t tw0 = globaltimer_ns();
+  uint64_t tw = tw0;
+  unsigned idle = 0;
+  for (;;) {
+    bool did = false;
+    if (!SEQ && kr < nch) {
+      const int need = CH * kr + CH - RR;
+      if (consumed < need) prog_read(from_c, consumed, complete);
+      if (consumed >= need) {
+        if (!(P.dbg_skip & 1u)) issue_chunk(kr);  // (timing experiments only: results invalid)
+        if (kr + C::PFC < nch) prefetch_chunk(kr + C::PFC);
+        cp_async_commit();
+        ++kr;
+        did = true;
+      }
+    }
+    if (ks < nch) {
+      const int need = min(n, CH * ks + CH);
+      if (complete < need) prog_read(from_c, consumed, complete);
+      if (complete >= need) {
+        if (!(P.dbg_skip & 1u)) store_chunk(ks);
+        ++ks;
+        did = true;
+      }
+    }
+    int nl;
+    if (SEQ || kr == nch) {
+      cp_async_wait<0>();
+      nl = n;
+    } else {
+      cp_async_wait<LAG>();  // chunks <= kr-1-LAG landed (this lane's copies)
+      nl = min(n, max(0, CH * (kr - LAG)));
+    }
+    const int ns = min(n, CH * ks);
     if (nl > landed || ns > stored) {
       landed = max(landed, nl);
       stored = max(stored, ns);
-      prog_publish(to_c, landed, stored);  // __syncwarp: every lane's copies landed
+      prog_publish(to_c, landed, stored, (P.dbg_skip & 2u) != 0);  // __syncwarp: every lane's copies landed
     }
-    if (!SEQ && k < nch) {
-      wait_for(consumed, complete, true, CH * k + CH - R);
-      issue_chunk(k);
-      if (k + C::PFC < nch) prefetch_chunk(k + C::PFC);
-    }
-    cp_async_commit();
-    const int js = k - SK;
-    if (js >= 0 && js < nch) {
-      wait_for(consumed, complete, false, min(n, CH * js + CH));
-      store_chunk(js);
+    if (ks == nch && landed == n) break;
+    if (did) {
+      idle = 0;
+    } else if ((++idle & 255u) == 0) {
+      const uint64_t now = globaltimer_ns();
+      if (idle == 256) tw = now;
+      else if (now - tw > P.spin_limit_ns) watchdog_trap(P.err);
     }
   }
+  (void)tw0;
   prog_publish(to_c, n, n);
 }
 
 // The compute warp of a band: the wavefront sweep (no staging instructions in the step).
-template <class C, bool RAGGED>
+// SRC (compile time): where the band's left border column comes from.
+template <class C, bool RAGGED, int SRC>
 __device__ __forceinline__ void wave_band(const StripParams& P, const long long task, const int w, const int t,
                                           unsigned char* const smem, unsigned char* const wsm, const uint32_t gen,
                                           const int sink) {
-  constexpr int K = C::K, CH = C::CH, R = C::R;
+  constexpr int K = C::K, CE = C::CE, RR = C::RR, SR = C::SR;
   constexpr uint32_t RS4 = 4u * C::RS;
   constexpr bool SEQ = C::SEQ;
   constexpr unsigned FULL = 0xffffffffu;
+  constexpr int BD = SRC == kSrcGlobal ? 1 : 3;  // border prefetch distance (blocks)
   const bool tracing = P.trace != nullptr;
   const unsigned long long t_task0 = tracing ? globaltimer_ns() : 0ull;
-  long long spin_cyc = 0, ev_cyc = 0, bp_cyc = 0, wait_cyc = 0;
+  long long spin_cyc = 0, wait_cyc = 0, bp_cyc = 0;
+  const bool relaxed = (P.dbg_skip & 2u) != 0;
 
   const BandGeo<C> g(P, task, wsm);
   const int n = g.n, p = g.p, band = g.band, c0 = g.c0, ws = g.ws;
@@ -309,20 +350,15 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
   const uint32_t s_prog = smem_u32(smem + 8);     // [4w]: rows consumed by warp w (shared source)
   const uint32_t s_bring = smem_u32(smem + 128);  // [w * BR * 8]: ring warp w -> w+1
 
-  // ---- border source (left), uniform per task
-  int src;
+  // ---- border source (left)
   const uint64_t* lin = nullptr;
   uint32_t lin_epoch = 0;
   bool lin_sys = false;
   if (band == 0) {
-    src = P.halo_in ? kSrcGlobal : kSrcPlain;
     lin = P.halo_in;
     lin_sys = true;
     lin_epoch = P.halo_epoch;
-  } else if (w > 0) {
-    src = kSrcSmem;
-  } else {
-    src = kSrcGlobal;
+  } else if (SRC == kSrcGlobal) {
     lin = P.xbuf + (pair * (P.nbands - 1) + band - 1) * xstride(n);
     lin_epoch = P.epoch;
   }
@@ -352,41 +388,42 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
   const int out_m = (ws - 1) - out_lane * K;  // the band's last column within the out lane
   const bool do_out = t == out_lane && sink != kSinkNone;
 
-  // ---- border blocks: lane j < CH of block q holds the entry of row CH*q + 1 + j
+  // ---- border blocks: lane j < CE of block q holds the entry of row CE*q + 1 + j
   auto load_block = [&](int q) -> uint64_t {  // synchronous (shared source / re-poll)
-    const int row = CH * q + 1 + t;
-    if (t >= CH || row > n) return 0ull;
-    if (src == kSrcGlobal) return lin_sys ? ld_relaxed_sys(lin + row) : ld_relaxed_gpu(lin + row);
-    if (src == kSrcSmem) return lds64_volatile(bring_in + 8u * (row & (C::BR - 1)));
+    const int row = CE * q + 1 + t;
+    if (t >= CE || row > n) return 0ull;
+    if constexpr (SRC == kSrcGlobal) return lin_sys ? ld_relaxed_sys(lin + row) : ld_relaxed_gpu(lin + row);
+    if constexpr (SRC == kSrcSmem) return lds64_volatile(bring_in + 8u * (row & (C::BR - 1)));
     return static_cast<uint32_t>(__ldg(colp + static_cast<long long>(row) * lds));
   };
-  // Global / plain sources: block q is copied by cp.async three blocks ahead (one commit group
-  // per event, so the event's wait covers it) into slot q & 3 of a shared ring: rows
-  // CH*q .. CH*q+CH+1 (global: 16-byte pairs (2k, 2k+1) through L2 only, never via L1 since the
-  // entries are polled; plain: the 4-byte values of score column c0-1).  No register holds an
-  // in-flight load across an event (a register move of one stalls the warp for the latency).
+  // Global / plain sources: block q is copied by cp.async BD blocks ahead (one commit group per
+  // event) into slot q & 3 of a shared ring -- a polled global source ONE block ahead (an older
+  // snapshot would add its age to the band-to-band lag), the plain input column three blocks
+  // ahead: rows CE*q .. CE*q+CE+1 (global: 16-byte pairs (2k, 2k+1) through L2 only, never via L1
+  // since the entries are polled; plain: the 4-byte values of score column c0-1).  No register
+  // holds an in-flight load across an event (a register move of one stalls for the latency).
   auto prefetch_block = [&](int q) {
-    const uint32_t slot = g.bpre + 8u * (CH + 2) * static_cast<uint32_t>(q & 3);
-    if (src == kSrcGlobal) {
-      const int row = CH * q + 2 * t;
-      cp_async16_cg_p(t <= CH / 2 && row <= n, slot + 16u * t, lin + row);
-    } else if (src == kSrcPlain) {
-      const int row = CH * q + 1 + t;
-      cp_async4_p(t < CH && row <= n, slot + 8u * (1 + t), colp + static_cast<long long>(row) * lds);
+    const uint32_t slot = g.bpre + 8u * (CE + 2) * static_cast<uint32_t>(q & 3);
+    if constexpr (SRC == kSrcGlobal) {
+      const int row = CE * q + 2 * t;
+      cp_async16_cg_p(t <= CE / 2 && row <= n, slot + 16u * t, lin + row);
+    } else if constexpr (SRC == kSrcPlain) {
+      const int row = CE * q + 1 + t;
+      cp_async4_p(t < CE && row <= n, slot + 8u * (1 + t), colp + static_cast<long long>(row) * lds);
     }
   };
   auto read_block = [&](int q) -> uint64_t {
-    const uint32_t slot = g.bpre + 8u * (CH + 2) * static_cast<uint32_t>(q & 3);
-    return t < CH ? lds64_volatile(slot + 8u * (1 + t)) : 0ull;
+    const uint32_t slot = g.bpre + 8u * (CE + 2) * static_cast<uint32_t>(q & 3);
+    return t < CE ? lds64_volatile(slot + 8u * (1 + t)) : 0ull;
   };
   auto block_ok = [&](uint64_t e, int q) -> bool {
-    const int row = CH * q + 1 + t;
+    const int row = CE * q + 1 + t;
     bool ok = true;
-    if (t < CH && row <= n) {
+    if (t < CE && row <= n) {
       const uint32_t hi = static_cast<uint32_t>(e >> 32);
-      if (src == kSrcGlobal)
+      if constexpr (SRC == kSrcGlobal)
         ok = hi == lin_epoch;
-      else if (src == kSrcSmem)
+      else if constexpr (SRC == kSrcSmem)
         ok = hi == (gen | static_cast<uint32_t>(row));
     }
     return __all_sync(FULL, ok) != 0;
@@ -397,12 +434,13 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
 #pragma unroll
   for (int m = 0; m < K; ++m) Pv[m] = (t * K + m < ws) ? __ldg(g.S + c0 + t * K + m) : 0;
   int Lprev = (t * K < ws) ? __ldg(g.S + c0 + t * K - 1) : 0;  // diag input of the first row
-  uint64_t e1 = src == kSrcSmem ? load_block(0) : 0ull;        // shared source: the next block's entries
-  if (src != kSrcSmem)
-    for (int q = 0; q < 3; ++q) prefetch_block(q);
-  cp_async_commit();  // three groups before event 0: event Q's wait completes block Q-3's group
-  cp_async_commit();
-  cp_async_commit();
+  uint64_t e1 = 0ull;                                           // shared source: the next block's entries
+  if constexpr (SRC == kSrcSmem) {
+    e1 = load_block(0);
+  } else {
+    for (int q = 0; q < BD; ++q) prefetch_block(q);
+    cp_async_commit();
+  }
 
   // SEQ: per-band substitution profile prof[x][t] = pack_m subst[x][b[c0-1+tK+m]] (int8 x K)
   const uint8_t* const A = SEQ ? P.seq_a + pair * P.psa : nullptr;
@@ -449,8 +487,9 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     }
   };
 
-  // one wavefront step s = CH*Q + j; ALL = every lane's row is in 1..n (no predicates)
-  auto step = [&](const int s, const int j, auto all_tag) {
+  // one wavefront step s (entry jj of the block's border window); ALL = every lane's row is in
+  // 1..n (no predicates)
+  auto step = [&](const int s, const int jj, auto all_tag) {
     constexpr bool ALL = decltype(all_tag)::value;
     const int r = s + 1 - t;  // this lane's row
     // ---- ref of this step's row (loaded last step) and the next row's loads
@@ -472,10 +511,10 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     } else {
 #pragma unroll
       for (int m = 0; m < K; ++m) rv[m] = rvn[m];
-      load_ref_row(laneR + static_cast<uint32_t>(r & (R - 1)) * RS4);  // ring row of row r+1
+      load_ref_row(laneR + static_cast<uint32_t>(r & (RR - 1)) * RS4);  // ring row of row r+1
     }
     // ---- left value: lane t-1's last column of this row, lane 0: the border entry
-    const int bval = __shfl_sync(FULL, static_cast<int>(static_cast<uint32_t>(cur)), j);
+    const int bval = __shfl_sync(FULL, static_cast<int>(static_cast<uint32_t>(cur)), jj);
     const int from_left = __shfl_up_sync(FULL, vlast, 1);
     const int L = (t == 0) ? bval : from_left;
     bool active = true;
@@ -494,7 +533,7 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
 #pragma unroll
       for (int m = 0; m < K; ++m) Pv[m] = __viaddmax_s32(L, negp[m], Y[m]);  // max(L - (m+1)p, Y_m)
       Lprev = L;
-      const uint32_t aS = laneS + static_cast<uint32_t>((r - 1) & (R - 1)) * RS4;
+      const uint32_t aS = laneS + static_cast<uint32_t>((r - 1) & (SR - 1)) * RS4;
       [&]<int... I>(std::integer_sequence<int, I...>) {
         (sts128_ring<16 * I>(aS, Pv[4 * I], Pv[4 * I + 1], Pv[4 * I + 2], Pv[4 * I + 3]), ...);
       }(std::make_integer_sequence<int, K / 4>{});
@@ -511,16 +550,15 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
   };
 
   const int nsteps = n + 31;  // compute steps 0 .. n+30
-  const int nblk = (nsteps + CH - 1) / CH;
+  const int nblk = (nsteps + CE - 1) / CE;
   for (int Q = 0; Q < nblk; ++Q) {
-    const int sig0 = Q * CH;
-    const long long c_ev0 = tracing ? clock64() : 0;
+    const int sig0 = Q * CE;
     // ---- event Q.  To the staging warp: ref rows <= sig0-30 consumed (lane 31 read row sig0-30
     // at step sig0-1), score rows <= sig0-31 complete (lane 31 wrote row sig0-31 at step sig0-1).
-    prog_publish(to_s, max(0, sig0 - 30), max(0, sig0 - 31));
+    prog_publish(to_s, max(0, sig0 - 30), max(0, sig0 - 31), relaxed);
     {
-      // this block reads ref rows <= sig0+CH+1 and rewrites score slots of rows <= sig0+CH
-      const int need_l = SEQ ? 0 : min(n, sig0 + CH + 1), need_s = sig0 + CH - R;
+      // this block reads ref rows <= sig0+CE+1 and rewrites score slots of rows <= sig0+CE
+      const int need_l = SEQ ? 0 : min(n, sig0 + CE + 1), need_s = sig0 + CE - SR;
       if (landed < need_l || stored < need_s) {
         const long long c0c = clock64();
         const uint64_t tw = globaltimer_ns();
@@ -533,18 +571,22 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
         wait_cyc += clock64() - c0c;
       }
     }
-    cp_async_commit();   // the border copies issued at event Q-1 (block Q+2)
-    cp_async_wait<2>();  // block Q's border entries landed
-    __syncwarp();        // cp.async landed by lanes 0..CH-1 visible to the warp
-    if (sig0 < nsteps) {
-      if (src == kSrcSmem) {
-        cur = e1;
-        e1 = load_block(Q + 1);
-      } else {
-        cur = read_block(Q);     // issued at event Q-3
-        prefetch_block(Q + 3);   // into the slot of block Q-1 (read at the previous event)
-      }
-      if (src != kSrcPlain && !block_ok(cur, Q)) {
+    if constexpr (SRC == kSrcSmem) {
+      cur = e1;
+      if (sig0 + CE < nsteps) e1 = load_block(Q + 1);
+      if (t == 0) sts32_volatile(prog_in, sig0);  // rows <= sig0 consumed (block Q-1 validated)
+    } else {
+      if (sig0 + CE * BD < nsteps) prefetch_block(Q + BD);
+      cp_async_commit();  // this event's border copy
+      if constexpr (BD == 1)
+        cp_async_wait<1>();  // every earlier group landed: block Q's border entries
+      else
+        cp_async_wait<3>();  // the groups of events <= Q-3 landed
+      __syncwarp();          // landed by lanes 0..CE-1, visible to the warp
+      cur = read_block(Q);
+    }
+    if constexpr (SRC != kSrcPlain) {
+      if (!block_ok(cur, Q)) {
         const long long c0c = clock64();
         const uint64_t tw = globaltimer_ns();
         unsigned spins = 0;
@@ -554,34 +596,38 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
         } while (!block_ok(cur, Q));
         spin_cyc += clock64() - c0c;
       }
-      if (src == kSrcSmem && t == 0) sts32_volatile(prog_in, sig0 + CH);  // rows <= sig0+CH consumed
-      if (sink_smem) {
-        // rows written in this block are <= sig0+CH; the slot of row x held row x-BR
-        const int need = sig0 + CH - C::BR;
-        if (need > bp_cache && need > (bp_cache = lds32_volatile(prog_out))) {
-          const long long c0c = clock64();
-          const uint64_t tw = globaltimer_ns();
-          while (need > (bp_cache = lds32_volatile(prog_out)))
-            if (globaltimer_ns() - tw > P.spin_limit_ns) watchdog_trap(P.err);
-          bp_cyc += clock64() - c0c;
-        }
+    }
+    if (sink_smem) {
+      // rows written in this block are <= sig0+CE; the slot of row x held row x-BR
+      const int need = sig0 + CE - C::BR;
+      if (need > bp_cache && need > (bp_cache = lds32_volatile(prog_out))) {
+        const long long c0c = clock64();
+        const uint64_t tw = globaltimer_ns();
+        while (need > (bp_cache = lds32_volatile(prog_out)))
+          if (globaltimer_ns() - tw > P.spin_limit_ns) watchdog_trap(P.err);
+        bp_cyc += clock64() - c0c;
       }
     }
     asm volatile("mov.u32 %0, 0;" : "=r"(tok)::"memory");  // the block's ref loads stay below
     if constexpr (!SEQ) {
-      if (Q == 0) load_ref_row(laneR + static_cast<uint32_t>((-t) & (R - 1)) * RS4);  // row 1-t
+      if (Q == 0) load_ref_row(laneR + static_cast<uint32_t>((-t) & (RR - 1)) * RS4);  // row 1-t
     }
-    if (tracing) ev_cyc += clock64() - c_ev0;
-    // ---- CH steps
-    if (sig0 >= 31 && sig0 + CH <= n) {
+    // ---- CE steps (two unrolled halves of CE/2)
+    if (sig0 >= 31 && sig0 + CE <= n) {
+#pragma unroll 1
+      for (int h = 0; h < CE; h += CE / 2) {
 #pragma unroll
-      for (int j = 0; j < CH; ++j) step(sig0 + j, j, std::true_type{});
+        for (int j = 0; j < CE / 2; ++j) step(sig0 + h + j, h + j, std::true_type{});
+      }
     } else {
+#pragma unroll 1
+      for (int h = 0; h < CE; h += CE / 2) {
 #pragma unroll
-      for (int j = 0; j < CH; ++j) step(sig0 + j, j, std::false_type{});
+        for (int j = 0; j < CE / 2; ++j) step(sig0 + h + j, h + j, std::false_type{});
+      }
     }
   }
-  prog_publish(to_s, n, n);  // every row consumed and complete
+  prog_publish(to_s, n, n, relaxed);  // every row consumed and complete
   if (tracing && t == 0 && task < P.trace_cap) {
     unsigned smid;
     asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
@@ -590,7 +636,7 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     e[1] = t_task0;
     e[2] = globaltimer_ns();
     e[3] = smid;
-    e[4] = static_cast<unsigned long long>(ev_cyc);
+    e[4] = 0;
     e[5] = static_cast<unsigned long long>(bp_cyc);
     e[6] = static_cast<unsigned long long>(spin_cyc);
     e[7] = static_cast<unsigned long long>(wait_cyc);
@@ -641,10 +687,22 @@ __global__ void __launch_bounds__(64 * C::NW, 1) nw_wave_kernel(const __grid_con
           sink = P.halo_out ? kSinkGlobal : kSinkNone;
         else
           sink = (w < NW - 1) ? kSinkSmem : kSinkGlobal;
-        if (full)
-          wave_band<C, false>(P, task, w, t, smem, wsm, gen, sink);
-        else
-          wave_band<C, true>(P, task, w, t, smem, wsm, gen, sink);
+        const int src = band == 0 ? (P.halo_in ? kSrcGlobal : kSrcPlain) : (w > 0 ? kSrcSmem : kSrcGlobal);
+        if (full) {
+          if (src == kSrcGlobal)
+            wave_band<C, false, kSrcGlobal>(P, task, w, t, smem, wsm, gen, sink);
+          else if (src == kSrcSmem)
+            wave_band<C, false, kSrcSmem>(P, task, w, t, smem, wsm, gen, sink);
+          else
+            wave_band<C, false, kSrcPlain>(P, task, w, t, smem, wsm, gen, sink);
+        } else {
+          if (src == kSrcGlobal)
+            wave_band<C, true, kSrcGlobal>(P, task, w, t, smem, wsm, gen, sink);
+          else if (src == kSrcSmem)
+            wave_band<C, true, kSrcSmem>(P, task, w, t, smem, wsm, gen, sink);
+          else
+            wave_band<C, true, kSrcPlain>(P, task, w, t, smem, wsm, gen, sink);
+        }
       }
     }
     __syncthreads();  // group end: every warp done (shared rings / progress words reusable)

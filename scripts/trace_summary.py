@@ -10,3 +10,6 @@ span = (t[:, 2].max() - t[:, 1].min()) / 1e3
 print(f"bands={len(t)} span={span:.0f}us band0: {tot[0]/n:.1f} cyc/row (events {t[0,4]/n:.1f}, cp-wait {t[0,7]/n:.1f}, spin {t[0,6]/n:.1f}); "
       f"mean: total {tot.mean()/n:.1f} events {(t[:,4]/n).mean():.1f} spin {(t[:,6]/n).mean():.1f} bp {(t[:,5]/n).mean():.1f}; "
       f"last band ends {(t[-1,2]-t[:,1].min())/1e3:.0f}us, band0 ends {(t[0,2]-t[:,1].min())/1e3:.0f}us")
+if t.shape[1] >= 12:
+    ph = t[:, 8:12] / n
+    print("event phases cyc/row (publish, staging wait, cp.async+sync, border+bp): band0", np.round(ph[0], 1).tolist(), "mean", np.round(ph.mean(0), 1).tolist())
