@@ -35,17 +35,18 @@ nw_status cuda_fail(cudaError_t e) {
 
 constexpr int64_t kMaxN = (int64_t{1} << 30) - 64;
 
-// tile -> K (columns per lane) of the wavefront kernel: band width W = 32 K.  The paper's b x b
-// tiles (16/32/64) are narrower than one warp's band; they map to the W = 128 kernel (the
-// default, measured fastest at n = 32768); tile 256 selects the W = 256 kernel.
+// tile -> K (columns per lane) of the wavefront kernel: band width W = 32 K.  The default
+// (tile 0) is the W = 256 kernel (measured fastest at n = 32768: one band per CTA, its compute,
+// ref-staging and store-staging warps on three SM sub-partitions); the paper's b x b tiles
+// (16/32/64) and 128 map to the W = 128 kernel (two bands per CTA).
 int tile_to_k(int32_t tile) {
   switch (tile) {
     case 0:
+    case 256: return 8;
     case 16:
     case 32:
     case 64:
     case 128: return 4;
-    case 256: return 8;
     default: return 0;
   }
 }
@@ -70,9 +71,9 @@ nw_status check_range(int64_t n, int32_t p) {
 // Kernel instances: K columns per lane, SEQ (ref generated from the sequences), NW warps
 // (bands) per CTA (DESIGN.md §4.3 sizes the rings).
 // v5 self-staging wavefront kernels (nw_wave.cuh)
-using WCfg8 = WaveCfg<8, false, 1>;   // tile 256: W = 256, one band per CTA
+using WCfg8 = WaveCfg<8, false, 1>;   // tile 0 / 256: W = 256, one band per CTA
 using WCfg8S = WaveCfg<8, true, 1>;
-using WCfg4 = WaveCfg<4, false, 2>;   // tile 0 / 16 .. 128: W = 128, two bands per CTA
+using WCfg4 = WaveCfg<4, false, 2>;   // tile 16 .. 128: W = 128, two bands per CTA
 using WCfg4S = WaveCfg<4, true, 2>;
 
 struct DevInfo {
@@ -86,7 +87,7 @@ cudaError_t setup_wave(int* occ) {
   cudaError_t e = cudaFuncSetAttribute(nw_wave_kernel<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        static_cast<int>(C::kSmem));
   if (e != cudaSuccess) return e;
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, nw_wave_kernel<C>, 64 * C::NW, C::kSmem);
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, nw_wave_kernel<C>, 32 * C::NWARPS, C::kSmem);
 }
 
 std::mutex g_mu;
@@ -239,13 +240,13 @@ nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* 
   w->ticket_next += static_cast<unsigned long long>(P.ngroups + grid);  // every CTA draws one extra ticket
   const unsigned g = static_cast<unsigned>(grid);
   if (K == 8 && !SEQ)
-    nw_wave_kernel<WCfg8><<<g, 64 * WCfg8::NW, WCfg8::kSmem, st>>>(P);
+    nw_wave_kernel<WCfg8><<<g, 32 * WCfg8::NWARPS, WCfg8::kSmem, st>>>(P);
   else if (K == 8)
-    nw_wave_kernel<WCfg8S><<<g, 64 * WCfg8S::NW, WCfg8S::kSmem, st>>>(P);
+    nw_wave_kernel<WCfg8S><<<g, 32 * WCfg8S::NWARPS, WCfg8S::kSmem, st>>>(P);
   else if (!SEQ)
-    nw_wave_kernel<WCfg4><<<g, 64 * WCfg4::NW, WCfg4::kSmem, st>>>(P);
+    nw_wave_kernel<WCfg4><<<g, 32 * WCfg4::NWARPS, WCfg4::kSmem, st>>>(P);
   else
-    nw_wave_kernel<WCfg4S><<<g, 64 * WCfg4S::NW, WCfg4S::kSmem, st>>>(P);
+    nw_wave_kernel<WCfg4S><<<g, 32 * WCfg4S::NWARPS, WCfg4S::kSmem, st>>>(P);
   NW_CU(cudaGetLastError());
   return NW_OK;
 }

@@ -66,7 +66,8 @@ struct WaveCfg {
   static constexpr int REF_WORDS = SEQ ? 0 : RR * RS;
   static constexpr int PROF_WORDS = SEQ ? 32 * 32 * (K / 4) : 0;
   static constexpr int BPRE_BYTES = 4 * 8 * (CE + 2);  // border prefetch ring: 4 blocks x (CE+2) entries
-  static constexpr int HDR_BYTES = 128;                // progress words: [0] compute -> staging, [8] staging -> compute
+  static constexpr int HDR_BYTES = 128;                // progress words: [0] compute -> staging, [8] ref -> compute, [16] store -> compute
+  static constexpr int NWARPS = 3 * NW;                // per band: compute, ref-staging and store-staging warps
   static constexpr size_t kWarpSmem = HDR_BYTES + 4ull * (REF_WORDS + SR * RS + PROF_WORDS) + BPRE_BYTES;
   static constexpr size_t kCtaHdr = 128 + static_cast<size_t>(NW - 1) * BR * 8;
   static constexpr size_t kSmem = kCtaHdr + NW * kWarpSmem;
@@ -134,6 +135,8 @@ __device__ __forceinline__ void st_entry_smem_p(bool pred, uint32_t a, uint32_t 
                : "memory");
 }
 
+enum : int { kRoleRef = 1, kRoleStore = 2 };  // staging-warp roles
+
 // Shared per-band geometry of the compute and staging warps.
 template <class C>
 struct BandGeo {
@@ -180,15 +183,16 @@ __device__ __forceinline__ void prog_read(uint32_t a, int& lo, int& hi) {
 // The staging warp of a band: ref rows in (8-row chunks of 4-byte cp.async, paced by the ring
 // space the compute warp has released), score rows out (LDS.32 + coalesced STG.32 once the compute
 // warp has completed them), L2 prefetch ahead of the ref stream.
-template <class C, bool RAGGED>
+template <class C, bool RAGGED, int ROLE>
 __device__ __forceinline__ void wave_stage(const StripParams& P, const long long task, const int t, unsigned char* const wsm) {
+  constexpr bool DO_REF = (ROLE & kRoleRef) != 0, DO_ST = (ROLE & kRoleStore) != 0;
   constexpr int K = C::K, CH = C::CH, RR = C::RR, SR = C::SR;
   constexpr uint32_t RS4 = 4u * C::RS;
   constexpr bool SEQ = C::SEQ;
   const BandGeo<C> g(P, task, wsm);
   const int n = g.n;
   const int nch = (n + CH - 1) / CH;
-  const uint32_t from_c = g.hdr, to_c = g.hdr + 8;
+  const uint32_t from_c = g.hdr, to_c = g.hdr + (DO_REF ? 8 : 16);
   uint32_t wmask = 0;  // RAGGED: bit i = word 32i+t of the row segment exists
 #pragma unroll
   for (int i = 0; i < K; ++i) wmask |= static_cast<uint32_t>(32 * i + t < g.ws) << i;
@@ -273,7 +277,7 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
   // with RR = 128 the ref stream runs about RR/2 rows ahead, so both waits are satisfiable
   // (no deadlock) and normally already satisfied.
   constexpr int LAG = 3;
-  int kr = SEQ ? nch : 0, ks = 0;
+  int kr = (SEQ || !DO_REF) ? nch : 0, ks = DO_ST ? 0 : nch;
   const uint64_t tw0 = globaltimer_ns();
   uint64_t tw = tw0;
   unsigned idle = 0;
@@ -283,7 +287,7 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
       const int need = CH * kr + CH - RR;
       if (consumed < need) prog_read(from_c, consumed, complete);
       if (consumed >= need) {
-        if (!(P.dbg_skip & 1u)) issue_chunk(kr);  // (timing experiments only: results invalid)
+        if (!(P.dbg_skip & 5u)) issue_chunk(kr);  // (timing experiments only: results invalid)
         if (kr + C::PFC < nch) prefetch_chunk(kr + C::PFC);
         cp_async_commit();
         ++kr;
@@ -294,26 +298,33 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
       const int need = min(n, CH * ks + CH);
       if (complete < need) prog_read(from_c, consumed, complete);
       if (complete >= need) {
-        if (!(P.dbg_skip & 1u)) store_chunk(ks);
+        if (!(P.dbg_skip & 9u)) store_chunk(ks);
         ++ks;
         did = true;
       }
     }
-    int nl;
-    if (SEQ || kr == nch) {
-      cp_async_wait<0>();
-      nl = n;
+    if constexpr (DO_REF) {
+      int nl;
+      if (SEQ || kr == nch) {
+        cp_async_wait<0>();
+        nl = n;
+      } else {
+        cp_async_wait<LAG>();  // chunks <= kr-1-LAG landed (this lane's copies)
+        nl = min(n, max(0, CH * (kr - LAG)));
+      }
+      if (nl > landed) {
+        landed = nl;
+        prog_publish(to_c, landed, 0, (P.dbg_skip & 2u) != 0);  // __syncwarp: every lane's copies landed
+      }
+      if (landed == n) break;
     } else {
-      cp_async_wait<LAG>();  // chunks <= kr-1-LAG landed (this lane's copies)
-      nl = min(n, max(0, CH * (kr - LAG)));
+      const int ns = min(n, CH * ks);
+      if (ns > stored) {
+        stored = ns;
+        prog_publish(to_c, stored, 0, (P.dbg_skip & 2u) != 0);
+      }
+      if (ks == nch) break;
     }
-    const int ns = min(n, CH * ks);
-    if (nl > landed || ns > stored) {
-      landed = max(landed, nl);
-      stored = max(stored, ns);
-      prog_publish(to_c, landed, stored, (P.dbg_skip & 2u) != 0);  // __syncwarp: every lane's copies landed
-    }
-    if (ks == nch && landed == n) break;
     if (did) {
       idle = 0;
     } else if ((++idle & 255u) == 0) {
@@ -323,7 +334,6 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
     }
   }
   (void)tw0;
-  prog_publish(to_c, n, n);
 }
 
 // The compute warp of a band: the wavefront sweep (no staging instructions in the step).
@@ -346,7 +356,7 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
   const int n = g.n, p = g.p, band = g.band, c0 = g.c0, ws = g.ws;
   const long long pair = g.pair;
   const long long lds = P.lds;
-  const uint32_t to_s = g.hdr, from_s = g.hdr + 8;
+  const uint32_t to_s = g.hdr, from_r = g.hdr + 8, from_t = g.hdr + 16;
   const uint32_t s_prog = smem_u32(smem + 8);     // [4w]: rows consumed by warp w (shared source)
   const uint32_t s_bring = smem_u32(smem + 128);  // [w * BR * 8]: ring warp w -> w+1
 
@@ -416,7 +426,8 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     const uint32_t slot = g.bpre + 8u * (CE + 2) * static_cast<uint32_t>(q & 3);
     return t < CE ? lds64_volatile(slot + 8u * (1 + t)) : 0ull;
   };
-  auto block_ok = [&](uint64_t e, int q) -> bool {
+  // number of leading rows of block q whose entries in e are valid (uniform)
+  auto leading_valid = [&](uint64_t e, int q) -> int {
     const int row = CE * q + 1 + t;
     bool ok = true;
     if (t < CE && row <= n) {
@@ -426,7 +437,8 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
       else if constexpr (SRC == kSrcSmem)
         ok = hi == (gen | static_cast<uint32_t>(row));
     }
-    return __all_sync(FULL, ok) != 0;
+    const unsigned bad = ~__ballot_sync(FULL, ok);
+    return bad ? __ffs(bad) - 1 : 32;
   };
 
   // ---- prologue: top border row, first border blocks
@@ -563,8 +575,10 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
         const long long c0c = clock64();
         const uint64_t tw = globaltimer_ns();
         unsigned spins = 0;
+        int unused;
         for (;;) {
-          prog_read(from_s, landed, stored);
+          if (landed < need_l) prog_read(from_r, landed, unused);
+          if (stored < need_s) prog_read(from_t, stored, unused);
           if (landed >= need_l && stored >= need_s) break;
           if ((++spins & 255u) == 0 && globaltimer_ns() - tw > P.spin_limit_ns) watchdog_trap(P.err);
         }
@@ -586,14 +600,16 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
       cur = read_block(Q);
     }
     if constexpr (SRC != kSrcPlain) {
-      if (!block_ok(cur, Q)) {
+      // the whole block must be published before its first step (a row-by-row re-poll at the
+      // producer's frontier costs one round trip per row: measured slower)
+      if (leading_valid(cur, Q) < CE) {
         const long long c0c = clock64();
         const uint64_t tw = globaltimer_ns();
         unsigned spins = 0;
         do {
           cur = load_block(Q);
           if ((++spins & 255u) == 0 && globaltimer_ns() - tw > P.spin_limit_ns) watchdog_trap(P.err);
-        } while (!block_ok(cur, Q));
+        } while (leading_valid(cur, Q) < CE);
         spin_cyc += clock64() - c0c;
       }
     }
@@ -644,23 +660,25 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
 }
 
 template <class C>
-__global__ void __launch_bounds__(64 * C::NW, 1) nw_wave_kernel(const __grid_constant__ StripParams P) {
+__global__ void __launch_bounds__(32 * C::NWARPS, 1) nw_wave_kernel(const __grid_constant__ StripParams P) {
   constexpr int NW = C::NW;
   extern __shared__ __align__(128) unsigned char smem[];
   const int t = threadIdx.x & 31;
-  const int wa = threadIdx.x >> 5;  // 0..NW-1 compute warps, NW..2NW-1 staging warps
+  const int wa = threadIdx.x >> 5;  // 0..NW-1 compute, NW..2NW-1 ref staging, 2NW..3NW-1 store staging
   const bool staging = wa >= NW;
-  const int w = staging ? wa - NW : wa;  // the band slot this warp serves
+  const int role = wa < NW ? 0 : (wa < 2 * NW ? kRoleRef : kRoleStore);
+  const int w = wa % NW;  // the band slot this warp serves
   // CTA header: [0] group ticket, [8 + 4w] consumer progress of warp w, [128..] border rings
   unsigned long long* const s_group = reinterpret_cast<unsigned long long*>(smem);
   const uint32_t s_prog = smem_u32(smem + 8);
   unsigned char* const wsm = smem + C::kCtaHdr + w * C::kWarpSmem;
   // shared border rings start invalid (tag 0xFFFFFFFF never equals gen | row, row < 2^30)
-  for (int i = threadIdx.x; i < (NW - 1) * C::BR; i += 64 * NW) reinterpret_cast<unsigned long long*>(smem + 128)[i] = ~0ull;
+  for (int i = threadIdx.x; i < (NW - 1) * C::BR; i += 32 * C::NWARPS) reinterpret_cast<unsigned long long*>(smem + 128)[i] = ~0ull;
   if (threadIdx.x < NW) sts32_volatile(s_prog + 4 * threadIdx.x, 0);
   if (!staging && t == 0) {  // band progress words
     st_release_cta_v2(smem_u32(wsm), 0u, 0u);
     st_release_cta_v2(smem_u32(wsm) + 8, 0u, 0u);
+    st_release_cta_v2(smem_u32(wsm) + 16, 0u, 0u);
   }
   __syncthreads();
 
@@ -675,11 +693,16 @@ __global__ void __launch_bounds__(64 * C::NW, 1) nw_wave_kernel(const __grid_con
     if (task < P.ntasks) {
       const int band = static_cast<int>(task % P.nbands);
       const bool full = band_ws(P.width, band, C::W) == C::W;
-      if (staging) {
+      if (role == kRoleRef) {
         if (full)
-          wave_stage<C, false>(P, task, t, wsm);
+          wave_stage<C, false, kRoleRef>(P, task, t, wsm);
         else
-          wave_stage<C, true>(P, task, t, wsm);
+          wave_stage<C, true, kRoleRef>(P, task, t, wsm);
+      } else if (role == kRoleStore) {
+        if (full)
+          wave_stage<C, false, kRoleStore>(P, task, t, wsm);
+        else
+          wave_stage<C, true, kRoleStore>(P, task, t, wsm);
       } else {
         const bool last_band = band == P.nbands - 1;
         int sink;
@@ -710,6 +733,7 @@ __global__ void __launch_bounds__(64 * C::NW, 1) nw_wave_kernel(const __grid_con
     if (!staging && t == 0) {
       st_release_cta_v2(smem_u32(wsm), 0u, 0u);
       st_release_cta_v2(smem_u32(wsm) + 8, 0u, 0u);
+      st_release_cta_v2(smem_u32(wsm) + 16, 0u, 0u);
     }
     __syncthreads();
     ++gcount;

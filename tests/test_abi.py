@@ -117,7 +117,7 @@ def test_host_entry_validation(L):
 
 
 def test_band_width_and_launch_counts():
-    assert nwb.nw_band_width(0) == 128 and nwb.nw_band_width(128) == 128 and nwb.nw_band_width(256) == 256
+    assert nwb.nw_band_width(0) == 256 and nwb.nw_band_width(128) == 128 and nwb.nw_band_width(256) == 256
     assert nwb.nw_band_width(16) == nwb.nw_band_width(32) == nwb.nw_band_width(64) == 128
     assert nwb.nw_band_width(7) == 0
     assert nwb.nw_launch_count(0, 32768, 0) == 1                     # one persistent launch

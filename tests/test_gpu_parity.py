@@ -45,7 +45,7 @@ def gpu_fill(score, ref, p, tile, fn=None, ld=None, offset=0):
 SIZES = [1, 2, 3, 15, 16, 17, 31, 32, 33, 63, 64, 65, 100, 127, 128, 129, 255, 256, 257, 1000, 1024]
 
 
-@pytest.mark.parametrize("tile", [0, 16, 256])
+@pytest.mark.parametrize("tile", [0, 16])
 @pytest.mark.parametrize("n", SIZES)
 def test_fill_sizes(n, tile):
     score, ref = inputs.make_problem(n, 10, seed=n)
@@ -60,7 +60,7 @@ def test_fill_families(family, p):
     if family == "borders":
         kw = {"family": "random", "border_seed": 99}
     score, ref = inputs.make_problem(n, p, seed=3, **kw)
-    for tile in (0, 256):
+    for tile in (0, 128):
         np.testing.assert_array_equal(gpu_fill(score, ref, p, tile), expect(score, ref, p))
 
 
@@ -99,7 +99,7 @@ def test_small_grids_deadlock_free(grid):
 
 def test_workspace_reuse_across_sizes():
     """Epoch tags keep stale band borders of earlier calls (other n, other tile) harmless."""
-    for n, tile in [(300, 0), (1000, 256), (129, 0), (2000, 16), (300, 256)]:
+    for n, tile in [(300, 0), (1000, 128), (129, 0), (2000, 16), (300, 128)]:
         score, ref = inputs.make_problem(n, 10, seed=n + tile)
         np.testing.assert_array_equal(gpu_fill(score, ref, 10, tile), expect(score, ref, 10))
 
@@ -122,7 +122,7 @@ def test_fill_host_e2e():
     np.testing.assert_array_equal(got, want)
 
 
-@pytest.mark.parametrize("B,n,tile", [(1, 64, 0), (5, 100, 16), (7, 257, 0), (33, 64, 64), (3, 2048, 0), (4, 700, 256)])
+@pytest.mark.parametrize("B,n,tile", [(1, 64, 0), (5, 100, 16), (7, 257, 0), (33, 64, 64), (3, 2048, 0), (4, 700, 128)])
 def test_batch(B, n, tile):
     probs = [inputs.make_problem(n, 10, seed=inputs.pair_seed(k)) for k in range(B)]
     S = torch.from_numpy(np.stack([s for s, _ in probs])).cuda()
@@ -150,7 +150,7 @@ def split_strips(score, ref, G, tile):
     return out
 
 
-@pytest.mark.parametrize("G,n,tile", [(2, 256, 0), (3, 500, 16), (4, 1024, 0), (8, 1000, 64), (3, 1111, 128), (2, 600, 256), (4, 1500, 256)])
+@pytest.mark.parametrize("G,n,tile", [(2, 256, 0), (3, 500, 16), (4, 1024, 0), (8, 1000, 64), (3, 1111, 128), (2, 600, 128), (4, 1500, 0)])
 def test_sharded_single_device(G, n, tile):
     """Config 5's protocol on one GPU: G strips launched in rank order on one stream, each
     pushing its right border into the next strip's halo (epoch-tagged entries)."""
@@ -192,7 +192,7 @@ def _stream_compare(s_dev, score_row0, ref, n, p, chunk=2048):
     st.close()
 
 
-@pytest.mark.parametrize("n,tile", [(16384, 256), (32768, 0)])
+@pytest.mark.parametrize("n,tile", [(16384, 128), (32768, 0)])
 def test_full_size_configs_bit_exact(n, tile):
     """BASELINE.json configs 2/3 at full size, in the launch configuration bench.py times:
     every cell against the streaming oracle."""
@@ -208,7 +208,7 @@ def test_full_size_configs_bit_exact(n, tile):
     _stream_compare(s_dev, score[0], ref, n, p)
 
 
-@pytest.mark.parametrize("tile", [0, 256])
+@pytest.mark.parametrize("tile", [0, 128])
 @pytest.mark.parametrize("n", [1, 5, 31, 64, 129, 1000, 4096])
 def test_fill_seq_next2(n, tile):
     """NEXT-2: ref generated on chip from (a, b, BLOSUM62) == nw_fill on the materialised ref."""
