@@ -10,5 +10,5 @@ timeout 400 python bench.py --steps 10 --warmup 3 --trace gpurun_out/trace_c3.np
 for t in 16 64 128; do timeout 200 python bench.py --config 2 --tile $t --steps 10 --no-cpu --e2e-steps 0 > gpurun_out/bench_c2_t$t.json 2>&1; tail -1 gpurun_out/bench_c2_t$t.json | cut -c1-400; done
 timeout 300 python bench.py --config 3 --variant diagonal --steps 3 --no-cpu --e2e-steps 0 > gpurun_out/bench_c3_diag.json 2>&1; tail -1 gpurun_out/bench_c3_diag.json | cut -c1-300
 timeout 300 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none -k regex:nw_ -c 6 --csv --log-file gpurun_out/launches_c3.csv python bench.py --steps 2 --warmup 3 --no-cpu --e2e-steps 0 > /dev/null 2>&1; echo ncu1_rc=$?
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:nw_strip -s 3 -c 1 -o gpurun_out/prof_c3 python bench.py --steps 1 --warmup 3 --no-cpu --e2e-steps 0 > gpurun_out/ncu_full.log 2>&1; echo ncu2_rc=$?; tail -3 gpurun_out/ncu_full.log
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:nw_wave -s 3 -c 1 -o gpurun_out/prof_c3 python bench.py --steps 1 --warmup 3 --no-cpu --e2e-steps 0 > gpurun_out/ncu_full.log 2>&1; echo ncu2_rc=$?; tail -3 gpurun_out/ncu_full.log
 timeout 300 python bench.py --config 3 --variant seq --steps 10 --no-cpu --e2e-steps 0 > gpurun_out/bench_c3_seq.json 2>&1; tail -1 gpurun_out/bench_c3_seq.json | cut -c1-400
