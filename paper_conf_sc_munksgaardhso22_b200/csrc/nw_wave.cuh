@@ -64,7 +64,7 @@ struct WaveCfg {
   static constexpr int BR = 256;                // shared border ring entries
   static constexpr int NL = (4 * W + 127) / 128 + 1;  // 128-byte lines touched by one row segment
   static constexpr int REF_WORDS = SEQ ? 0 : RR * RS;
-  static constexpr int PROF_WORDS = SEQ ? 32 * 32 * (K / 4) : 0;
+  static constexpr int PROF_WORDS = SEQ ? 32 * 32 * K : 0;  // int32 prof[x][lane][K] (+2p, gap-normalised)
   static constexpr int BPRE_BYTES = 4 * 8 * (CE + 2);  // border prefetch ring: 4 blocks x (CE+2) entries
   static constexpr int HDR_BYTES = 128;                // progress words: [0] compute -> staging, [8] ref -> compute, [16] store -> compute
   static constexpr int NWARPS = 3 * NW;                // per band: compute, ref-staging and store-staging warps
@@ -73,7 +73,8 @@ struct WaveCfg {
   static constexpr size_t kSmem = kCtaHdr + NW * kWarpSmem;
   static_assert(K == 4 || K == 8, "K/4 LDS.128 per step");
   static_assert((RS * 4 / 16) % 8 == DELTA, "bank-group shift");
-  static_assert(kWarpSmem % 16 == 0 && kCtaHdr % 16 == 0, "16-byte aligned rings");
+  static_assert(kWarpSmem % 32 == 0 && kCtaHdr % 32 == 0 && (HDR_BYTES + 4 * (REF_WORDS + SR * RS)) % 32 == 0,
+                "32-byte aligned rings (the profile's half-swap flips address bit 4)");
   static_assert(NL <= 32 && NW <= 8, "geometry");
   static_assert(RR % CH == 0 && (RR & (RR - 1)) == 0 && SR % CH == 0 && (SR & (SR - 1)) == 0 && RR >= 64 && SR >= 64,
                 "rings of whole chunks, powers of two, large enough for the staging schedule");
@@ -96,6 +97,10 @@ __device__ __forceinline__ int lds32_imm(uint32_t a) {
   int v;
   asm volatile("ld.shared.b32 %0, [%1+%2];" : "=r"(v) : "r"(a), "n"(OFF) : "memory");
   return v;
+}
+template <int OFF>
+__device__ __forceinline__ void sts32_imm(uint32_t a, int v) {
+  asm volatile("st.shared.b32 [%0+%2], %1;" ::"r"(a), "r"(v), "n"(OFF) : "memory");
 }
 template <int OFF>
 __device__ __forceinline__ void stg32_imm_p(bool p, uint64_t g, int v) {
@@ -199,20 +204,6 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
   const uint64_t ldr4 = 4ull * static_cast<uint64_t>(P.ldr), lds4 = 4ull * static_cast<uint64_t>(P.lds);
   const uint64_t gR0 = SEQ ? 0ull : reinterpret_cast<uint64_t>(g.Rf + g.c0 + t);  // (row 0, word t) of the ref segment
   const uint64_t gS0 = reinterpret_cast<uint64_t>(g.S + g.c0 + t);
-  const unsigned long long spin = P.spin_limit_ns;
-  auto wait_for = [&](int& cache_lo, int& cache_hi, bool want_lo, int need) {
-    // cached progress of the compute warp: lo = ref rows consumed, hi = score rows complete
-    int v = want_lo ? cache_lo : cache_hi;
-    if (v >= need) return;
-    const uint64_t tw = globaltimer_ns();
-    unsigned spins = 0;
-    for (;;) {
-      prog_read(from_c, cache_lo, cache_hi);
-      v = want_lo ? cache_lo : cache_hi;
-      if (v >= need) return;
-      if ((++spins & 255u) == 0 && globaltimer_ns() - tw > spin) watchdog_trap(P.err);
-    }
-  };
   int consumed = 0, complete = 0;  // cached compute-warp progress
   int landed = 0, stored = 0;      // published to the compute warp
   // chunk k of ref: rows CH*k+1 .. CH*k+CH (row i of the chunk: K copies per lane)
@@ -247,6 +238,11 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
       }
     }
   };
+  // the compute warp's ring holds the gap-normalised S' = S + (i + j) p: the
+  // store converts back, one IADD3 per value: S = S' - r p - (c0 + 32 I + t) p
+  int colp[K];
+#pragma unroll
+  for (int I = 0; I < K; ++I) colp[I] = (g.c0 + 32 * I + t) * g.p;
   auto store_chunk = [&](int k) {
     int v[CH][K];
 #pragma unroll
@@ -258,6 +254,9 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
 #pragma unroll
     for (int i = 0; i < CH; ++i) {
       const int ro = CH * k + 1 + i;
+      const int rp = ro * g.p;
+#pragma unroll
+      for (int I = 0; I < K; ++I) v[i][I] = v[i][I] - rp - colp[I];
       const uint64_t ga = gS0 + static_cast<uint64_t>(static_cast<long long>(ro)) * lds4;
       if constexpr (!RAGGED) {
         [&]<int... I>(std::integer_sequence<int, I...>) { (stg32_imm_p<128 * I>(ro <= n, ga, v[i][I]), ...); }(std::make_integer_sequence<int, K>{});
@@ -338,7 +337,9 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
 
 // The compute warp of a band: the wavefront sweep (no staging instructions in the step).
 // SRC (compile time): where the band's left border column comes from.
-template <class C, bool RAGGED, int SRC>
+// HALO_OUT (compile time): the band pushes its last column into a strip halo, whose entries
+// hold the true S (nw.h), not the kernel's gap-normalised S'.
+template <class C, bool RAGGED, int SRC, bool HALO_OUT>
 __device__ __forceinline__ void wave_band(const StripParams& P, const long long task, const int w, const int t,
                                           unsigned char* const smem, unsigned char* const wsm, const uint32_t gen,
                                           const int sink) {
@@ -442,10 +443,11 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
   };
 
   // ---- prologue: top border row, first border blocks
+  // gap-normalised values S' = S + (i + j) p; row 0: S'(0, j) = S(0, j) + j p
   int Pv[K];
 #pragma unroll
-  for (int m = 0; m < K; ++m) Pv[m] = (t * K + m < ws) ? __ldg(g.S + c0 + t * K + m) : 0;
-  int Lprev = (t * K < ws) ? __ldg(g.S + c0 + t * K - 1) : 0;  // diag input of the first row
+  for (int m = 0; m < K; ++m) Pv[m] = (t * K + m < ws) ? __ldg(g.S + c0 + t * K + m) + (c0 + t * K + m) * p : 0;
+  int Lprev = (t * K < ws) ? __ldg(g.S + c0 + t * K - 1) + (c0 + t * K - 1) * p : 0;  // diag input of the first row
   uint64_t e1 = 0ull;                                           // shared source: the next block's entries
   if constexpr (SRC == kSrcSmem) {
     e1 = load_block(0);
@@ -454,33 +456,30 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     cp_async_commit();
   }
 
-  // SEQ: per-band substitution profile prof[x][t] = pack_m subst[x][b[c0-1+tK+m]] (int8 x K)
+  // SEQ: per-band substitution profile prof[x][t][m] = subst[x][b[c0-1+tK+m]] + 2p (int32, the
+  // diagonal move of the gap-normalised recurrence).  K = 8: lane t's two 16-byte halves are
+  // swapped when bit 2 of t is set, so the 8 lanes of an LDS.128 phase cover all 32 banks.
   const uint8_t* const A = SEQ ? P.seq_a + pair * P.psa : nullptr;
   int a_cur = 0, a_nxt = 0;  // residues of this lane's current / next row (software pipeline)
+  const uint32_t sw = K == 8 ? ((t >> 2) & 1u) : 0u;
   if constexpr (SEQ) {
-    uint32_t* const prof = reinterpret_cast<uint32_t*>(wsm + (g.prof - g.hdr));
+    int* const prof = reinterpret_cast<int*>(wsm + (g.prof - g.hdr));
     const uint8_t* const Bq = P.seq_b + pair * P.psb;
     int bj[K];
 #pragma unroll
     for (int m = 0; m < K; ++m) bj[m] = (t * K + m < ws) ? (Bq[c0 - 1 + t * K + m] & 31) : 0;
     for (int x = 0; x < 32; ++x) {
 #pragma unroll
-      for (int q = 0; q < K / 4; ++q) {
-        uint32_t wv = 0;
-#pragma unroll
-        for (int m = 0; m < 4; ++m) wv |= static_cast<uint32_t>(static_cast<uint8_t>(P.subst[x * 32 + bj[4 * q + m]])) << (8 * m);
-        prof[(x * 32 + t) * (K / 4) + q] = wv;
-      }
+      for (int m = 0; m < K; ++m)
+        prof[(x * 32 + t) * K + 4 * ((m >> 2) ^ sw) + (m & 3)] = static_cast<int>(P.subst[x * 32 + bj[m]]) + 2 * p;
     }
     a_cur = A[min(max(-t, 0), n - 1)] & 31;     // row 1-t
     a_nxt = A[min(max(1 - t, 0), n - 1)] & 31;  // row 2-t
     __syncwarp();
   }
-  const uint32_t profA = g.prof + 4u * (K / 4) * t;
+  const uint32_t profA = opaque(g.prof + 4u * K * t + 16u * sw);
 
-  int negp[K];  // -(m+1) p
-#pragma unroll
-  for (int m = 0; m < K; ++m) negp[m] = static_cast<int>(opaque(static_cast<uint32_t>(-(m + 1) * p)));
+  const int p2 = 2 * p;
   uint32_t tok = 0;  // produced after each event's acquire, consumed by the ref loads
   int rvn[K];        // ref of the lane's NEXT row (loaded one step ahead)
 #pragma unroll
@@ -488,6 +487,11 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
   int bp_cache = 0;            // last consumer progress read (back-pressure, shared sink)
   int landed = 0, stored = 0;  // cached staging-warp progress
   uint64_t cur = 0ull;
+  int curv = 0;  // lane j < CE: S' of the border entry of row CE*Q+1+j (the current block)
+  // band 0's border (score column 0 or a strip halo) holds the true S: S'(r, 0) = S(r, 0) + r p
+  const bool conv_in = SRC == kSrcPlain || (SRC == kSrcGlobal && band == 0);
+  // HALO_OUT: S(r, c_last) = S'(r, c_last) - (r + c_last) p, c_last = c0 + ws - 1
+  const int out_adj = HALO_OUT ? (c0 + ws - 1 + 1 - out_lane) * p : 0;  // + s p = (r + c_last) p at step s
   int vlast = Pv[K - 1];
   const uint32_t laneR = opaque(g.refR + 16u * (K / 4) * t), laneS = opaque(g.scR + 16u * (K / 4) * t);
   auto load_ref_row = [&](uint32_t a) {  // K/4 LDS.128 of this lane's K ref values
@@ -507,43 +511,51 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     // ---- ref of this step's row (loaded last step) and the next row's loads
     int rv[K];
     if constexpr (SEQ) {
-      uint32_t pw[K / 4];
+      const uint32_t a0 = profA + (static_cast<uint32_t>(a_cur) << (7 + (K == 8 ? 3 : 2)));  // + a * 32 lanes * 4K bytes
+      const int4 u = lds128_tok<0>(a0, tok);
+      rv[0] = u.x, rv[1] = u.y, rv[2] = u.z, rv[3] = u.w;
       if constexpr (K == 8) {
-        uint32_t lo, hi;
-        asm("ld.shared.v2.b32 {%0, %1}, [%2];" : "=r"(lo), "=r"(hi) : "r"(profA + 256u * a_cur));
-        pw[0] = lo;
-        pw[K / 4 - 1] = hi;
-      } else {
-        asm("ld.shared.b32 %0, [%1];" : "=r"(pw[0]) : "r"(profA + 128u * a_cur));
+        const int4 v = lds128_tok<0>(a0 ^ 16u, tok);
+        rv[4] = v.x, rv[5] = v.y, rv[6] = v.z, rv[7] = v.w;
       }
-#pragma unroll
-      for (int m = 0; m < K; ++m) rv[m] = prmt_sext(pw[m / 4], 0x8880u + 0x1111u * (m & 3));
       a_cur = a_nxt;
       a_nxt = __ldg(A + min(max(r + 1, 0), n - 1)) & 31;  // residue of row r+2
     } else {
+      // ref' = ref + 2p (the diagonal move of the gap-normalised recurrence); off the
+      // recurrence's critical path (the row was loaded one step ahead)
 #pragma unroll
-      for (int m = 0; m < K; ++m) rv[m] = rvn[m];
+      for (int m = 0; m < K; ++m) rv[m] = rvn[m] + p2;
       load_ref_row(laneR + static_cast<uint32_t>(r & (RR - 1)) * RS4);  // ring row of row r+1
     }
     // ---- left value: lane t-1's last column of this row, lane 0: the border entry
-    const int bval = __shfl_sync(FULL, static_cast<int>(static_cast<uint32_t>(cur)), jj);
+    const int bval = __shfl_sync(FULL, curv, jj);
     const int from_left = __shfl_up_sync(FULL, vlast, 1);
     const int L = (t == 0) ? bval : from_left;
     bool active = true;
     if (!ALL) active = r >= 1 && r <= n;
     if (active) {
-      int Y[K];
-      {
-        int d = Lprev;
+      // gap-normalised cell: S'(r,j) = max(S'(r-1,j-1) + ref'(r,j), S'(r-1,j), S'(r,j-1))
+      // x_m = max(diag + ref', up): one DPX each; the row's left chain is a plain prefix max
+      // (depth 4 with 3-input max) and the left value L enters with one max per cell.
+      int x[K];
+      x[0] = __viaddmax_s32(Lprev, rv[0], Pv[0]);
 #pragma unroll
-        for (int m = 0; m < K; ++m) {
-          const int x = __viaddmax_s32(Pv[m], -p, d + rv[m]);  // max(up - p, diag + ref)
-          Y[m] = m == 0 ? x : __viaddmax_s32(Y[m - 1], -p, x);
-          d = Pv[m];
-        }
+      for (int m = 1; m < K; ++m) x[m] = __viaddmax_s32(Pv[m - 1], rv[m], Pv[m]);
+      int Y[K];
+      Y[0] = x[0];
+      Y[1] = max(x[0], x[1]);
+      if constexpr (K >= 4) {
+        Y[2] = __vimax3_s32(x[0], x[1], x[2]);
+        Y[3] = __vimax3_s32(Y[1], x[2], x[3]);
+      }
+      if constexpr (K == 8) {
+        Y[4] = __vimax3_s32(Y[2], x[3], x[4]);
+        Y[5] = __vimax3_s32(Y[3], x[4], x[5]);
+        Y[6] = __vimax3_s32(Y[4], x[5], x[6]);
+        Y[7] = __vimax3_s32(Y[5], x[6], x[7]);
       }
 #pragma unroll
-      for (int m = 0; m < K; ++m) Pv[m] = __viaddmax_s32(L, negp[m], Y[m]);  // max(L - (m+1)p, Y_m)
+      for (int m = 0; m < K; ++m) Pv[m] = max(L, Y[m]);
       Lprev = L;
       const uint32_t aS = laneS + static_cast<uint32_t>((r - 1) & (SR - 1)) * RS4;
       [&]<int... I>(std::integer_sequence<int, I...>) {
@@ -554,6 +566,7 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
 #pragma unroll
         for (int m = 0; m < K - 1; ++m) vo = out_m == m ? Pv[m] : vo;
       }
+      if constexpr (HALO_OUT) vo -= out_adj + s * p;
       st_entry_smem_p(do_out && sink_smem, bring_out + 8u * (r & (C::BR - 1)), static_cast<uint32_t>(vo), gen | static_cast<uint32_t>(r));
       st_entry_gpu_p(do_out && sink_gpu, lout + r, static_cast<uint32_t>(vo), lout_tag);
       st_entry_sys_p(do_out && sink_sys, lout + r, static_cast<uint32_t>(vo), lout_tag);
@@ -613,6 +626,8 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
         spin_cyc += clock64() - c0c;
       }
     }
+    curv = static_cast<int>(static_cast<uint32_t>(cur));
+    if (conv_in) curv += (CE * Q + 1 + t) * p;
     if (sink_smem) {
       // rows written in this block are <= sig0+CE; the slot of row x held row x-BR
       const int need = sig0 + CE - C::BR;
@@ -711,20 +726,28 @@ __global__ void __launch_bounds__(32 * C::NWARPS, 1) nw_wave_kernel(const __grid
         else
           sink = (w < NW - 1) ? kSinkSmem : kSinkGlobal;
         const int src = band == 0 ? (P.halo_in ? kSrcGlobal : kSrcPlain) : (w > 0 ? kSrcSmem : kSrcGlobal);
-        if (full) {
+        const bool halo_out = last_band && P.halo_out;  // validated: such a band is full width
+        if (halo_out) {
           if (src == kSrcGlobal)
-            wave_band<C, false, kSrcGlobal>(P, task, w, t, smem, wsm, gen, sink);
+            wave_band<C, false, kSrcGlobal, true>(P, task, w, t, smem, wsm, gen, sink);
           else if (src == kSrcSmem)
-            wave_band<C, false, kSrcSmem>(P, task, w, t, smem, wsm, gen, sink);
+            wave_band<C, false, kSrcSmem, true>(P, task, w, t, smem, wsm, gen, sink);
           else
-            wave_band<C, false, kSrcPlain>(P, task, w, t, smem, wsm, gen, sink);
+            wave_band<C, false, kSrcPlain, true>(P, task, w, t, smem, wsm, gen, sink);
+        } else if (full) {
+          if (src == kSrcGlobal)
+            wave_band<C, false, kSrcGlobal, false>(P, task, w, t, smem, wsm, gen, sink);
+          else if (src == kSrcSmem)
+            wave_band<C, false, kSrcSmem, false>(P, task, w, t, smem, wsm, gen, sink);
+          else
+            wave_band<C, false, kSrcPlain, false>(P, task, w, t, smem, wsm, gen, sink);
         } else {
           if (src == kSrcGlobal)
-            wave_band<C, true, kSrcGlobal>(P, task, w, t, smem, wsm, gen, sink);
+            wave_band<C, true, kSrcGlobal, false>(P, task, w, t, smem, wsm, gen, sink);
           else if (src == kSrcSmem)
-            wave_band<C, true, kSrcSmem>(P, task, w, t, smem, wsm, gen, sink);
+            wave_band<C, true, kSrcSmem, false>(P, task, w, t, smem, wsm, gen, sink);
           else
-            wave_band<C, true, kSrcPlain>(P, task, w, t, smem, wsm, gen, sink);
+            wave_band<C, true, kSrcPlain, false>(P, task, w, t, smem, wsm, gen, sink);
         }
       }
     }
