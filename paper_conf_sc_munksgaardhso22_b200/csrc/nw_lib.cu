@@ -38,7 +38,7 @@ constexpr int64_t kMaxN = (int64_t{1} << 30) - 64;
 // tile -> K (columns per lane) of the wavefront kernel: band width W = 32 K.  The default
 // (tile 0) is the W = 256 kernel (measured fastest at n = 32768: one band per CTA, its compute,
 // ref-staging and store-staging warps on three SM sub-partitions); the paper's b x b tiles
-// (16/32/64) and 128 map to the W = 128 kernel (two bands per CTA).
+// (16/32/64) and 128 map to the W = 128 kernel (two bands per CTA, one staging warp per band).
 int tile_to_k(int32_t tile) {
   switch (tile) {
     case 0:
@@ -71,10 +71,10 @@ nw_status check_range(int64_t n, int32_t p) {
 // Kernel instances: K columns per lane, SEQ (ref generated from the sequences), NW warps
 // (bands) per CTA (DESIGN.md §4.3 sizes the rings).
 // v5 self-staging wavefront kernels (nw_wave.cuh)
-using WCfg8 = WaveCfg<8, false, 1>;   // tile 0 / 256: W = 256, one band per CTA
-using WCfg8S = WaveCfg<8, true, 1>;
-using WCfg4 = WaveCfg<4, false, 2>;   // tile 16 .. 128: W = 128, two bands per CTA
-using WCfg4S = WaveCfg<4, true, 2>;
+using WCfg8 = WaveCfg<8, false, 1, 2>;   // tile 0 / 256: W = 256, one band per CTA, ref + store warps
+using WCfg8S = WaveCfg<8, true, 1, 2>;
+using WCfg4 = WaveCfg<4, false, 2, 1>;   // tile 16 .. 128: W = 128, two bands per CTA
+using WCfg4S = WaveCfg<4, true, 2, 1>;
 
 struct DevInfo {
   bool init = false;
@@ -221,6 +221,11 @@ nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* 
       return e ? static_cast<unsigned>(std::strtoul(e, nullptr, 0)) : 0u;
     }();
     P.dbg_skip = dbg;
+    static const unsigned sleep_ns = [] {
+      const char* e = std::getenv("NW_STAGE_SLEEP_NS");
+      return e ? static_cast<unsigned>(std::strtoul(e, nullptr, 0)) : 0u;
+    }();
+    P.stage_sleep_ns = sleep_ns;
   }
   P.trace = g_trace;
   P.trace_cap = g_trace_cap;

@@ -49,9 +49,13 @@
 
 namespace nwb200 {
 
-template <int K_, bool SEQ_, int NW_>
+// K columns per lane (band width W = 32 K), SEQ (ref generated from the sequences), NW bands
+// (compute warps) per CTA, SPB staging warps per band (1: one warp moves ref in and score out;
+// 2: separate ref and store warps).  Warp w runs on SM sub-partition w % 4: the compute warps
+// take sub-partitions 0..NW-1 and the staging warps the others (NW * (1 + SPB) <= 4).
+template <int K_, bool SEQ_, int NW_, int SPB_>
 struct WaveCfg {
-  static constexpr int K = K_, NW = NW_;
+  static constexpr int K = K_, NW = NW_, SPB = SPB_;
   static constexpr bool SEQ = SEQ_;
   static constexpr int W = 32 * K;
   static constexpr int CH = 8;                  // staging chunk (rows)
@@ -67,7 +71,7 @@ struct WaveCfg {
   static constexpr int PROF_WORDS = SEQ ? 32 * 32 * K : 0;  // int32 prof[x][lane][K] (+2p, gap-normalised)
   static constexpr int BPRE_BYTES = 4 * 8 * (CE + 2);  // border prefetch ring: 4 blocks x (CE+2) entries
   static constexpr int HDR_BYTES = 128;                // progress words: [0] compute -> staging, [8] ref -> compute, [16] store -> compute
-  static constexpr int NWARPS = 3 * NW;                // per band: compute, ref-staging and store-staging warps
+  static constexpr int NWARPS = NW * (1 + SPB);        // per band: a compute warp and SPB staging warps
   static constexpr size_t kWarpSmem = HDR_BYTES + 4ull * (REF_WORDS + SR * RS + PROF_WORDS) + BPRE_BYTES;
   static constexpr size_t kCtaHdr = 128 + static_cast<size_t>(NW - 1) * BR * 8;
   static constexpr size_t kSmem = kCtaHdr + NW * kWarpSmem;
@@ -75,7 +79,7 @@ struct WaveCfg {
   static_assert((RS * 4 / 16) % 8 == DELTA, "bank-group shift");
   static_assert(kWarpSmem % 32 == 0 && kCtaHdr % 32 == 0 && (HDR_BYTES + 4 * (REF_WORDS + SR * RS)) % 32 == 0,
                 "32-byte aligned rings (the profile's half-swap flips address bit 4)");
-  static_assert(NL <= 32 && NW <= 8, "geometry");
+  static_assert(NL <= 32 && NW <= 8 && (SPB == 1 || SPB == 2) && NWARPS <= 4, "geometry: one warp per sub-partition");
   static_assert(RR % CH == 0 && (RR & (RR - 1)) == 0 && SR % CH == 0 && (SR & (SR - 1)) == 0 && RR >= 64 && SR >= 64,
                 "rings of whole chunks, powers of two, large enough for the staging schedule");
 };
@@ -84,6 +88,15 @@ struct WaveCfg {
 template <int OFF>
 __device__ __forceinline__ void cp_async4_imm(uint32_t dst, uint64_t src) {
   asm volatile("cp.async.ca.shared.global [%0+%2], [%1+%2], 4;" ::"r"(dst), "l"(src), "n"(OFF) : "memory");
+}
+template <int DOFF, int SOFF>
+__device__ __forceinline__ void cp_async4_imm2(uint32_t dst, uint64_t src) {
+  asm volatile("cp.async.ca.shared.global [%0+%2], [%1+%3], 4;" ::"r"(dst), "l"(src), "n"(DOFF), "n"(SOFF) : "memory");
+}
+// one row: K 4-byte copies / K 4-byte shared loads at compile-time offsets DBASE + 128 I
+template <int DBASE, int K>
+__device__ __forceinline__ void cp_row(uint32_t d0, uint64_t src) {
+  [&]<int... I>(std::integer_sequence<int, I...>) { (cp_async4_imm2<DBASE + 128 * I, 128 * I>(d0, src), ...); }(std::make_integer_sequence<int, K>{});
 }
 template <int OFF>
 __device__ __forceinline__ void cp_async4_imm_p(bool p, uint32_t dst, uint64_t src) {
@@ -98,9 +111,17 @@ __device__ __forceinline__ int lds32_imm(uint32_t a) {
   asm volatile("ld.shared.b32 %0, [%1+%2];" : "=r"(v) : "r"(a), "n"(OFF) : "memory");
   return v;
 }
+template <int DBASE, int K>
+__device__ __forceinline__ void lds_row(uint32_t a0, int* v) {
+  [&]<int... I>(std::integer_sequence<int, I...>) { ((v[I] = lds32_imm<DBASE + 128 * I>(a0)), ...); }(std::make_integer_sequence<int, K>{});
+}
 template <int OFF>
 __device__ __forceinline__ void sts32_imm(uint32_t a, int v) {
   asm volatile("st.shared.b32 [%0+%2], %1;" ::"r"(a), "r"(v), "n"(OFF) : "memory");
+}
+template <int OFF>
+__device__ __forceinline__ void stg32_imm(uint64_t g, int v) {
+  asm volatile("st.global.b32 [%0+%2], %1;" ::"l"(g), "r"(v), "n"(OFF) : "memory");
 }
 template <int OFF>
 __device__ __forceinline__ void stg32_imm_p(bool p, uint64_t g, int v) {
@@ -121,21 +142,20 @@ template <int OFF>
 __device__ __forceinline__ void sts128_ring(uint32_t a, int x, int y, int z, int w) {
   asm volatile("st.shared.v4.b32 [%0+%5], {%1, %2, %3, %4};" ::"r"(a), "r"(x), "r"(y), "r"(z), "r"(w), "n"(OFF));
 }
+// border-entry stores {value, tag}: v2.b32 straight from the value register (a 64-bit temporary
+// register pair reused step after step made every store wait for the previous one's operand read)
 __device__ __forceinline__ void st_entry_gpu_p(bool pred, uint64_t* p, uint32_t lo, uint32_t hi) {
-  asm volatile("{ .reg .pred q; .reg .b64 e; setp.ne.b32 q, %0, 0; mov.b64 e, {%2, %3}; @q st.relaxed.gpu.global.b64 [%1], e; }" ::"r"(
-                   static_cast<int>(pred)),
+  asm volatile("{ .reg .pred q; setp.ne.b32 q, %0, 0; @q st.relaxed.gpu.global.v2.b32 [%1], {%2, %3}; }" ::"r"(static_cast<int>(pred)),
                "l"(p), "r"(lo), "r"(hi)
                : "memory");
 }
 __device__ __forceinline__ void st_entry_sys_p(bool pred, uint64_t* p, uint32_t lo, uint32_t hi) {
-  asm volatile("{ .reg .pred q; .reg .b64 e; setp.ne.b32 q, %0, 0; mov.b64 e, {%2, %3}; @q st.relaxed.sys.global.b64 [%1], e; }" ::"r"(
-                   static_cast<int>(pred)),
+  asm volatile("{ .reg .pred q; setp.ne.b32 q, %0, 0; @q st.relaxed.sys.global.v2.b32 [%1], {%2, %3}; }" ::"r"(static_cast<int>(pred)),
                "l"(p), "r"(lo), "r"(hi)
                : "memory");
 }
 __device__ __forceinline__ void st_entry_smem_p(bool pred, uint32_t a, uint32_t lo, uint32_t hi) {
-  asm volatile("{ .reg .pred q; .reg .b64 e; setp.ne.b32 q, %0, 0; mov.b64 e, {%2, %3}; @q st.volatile.shared.b64 [%1], e; }" ::"r"(
-                   static_cast<int>(pred)),
+  asm volatile("{ .reg .pred q; setp.ne.b32 q, %0, 0; @q st.volatile.shared.v2.b32 [%1], {%2, %3}; }" ::"r"(static_cast<int>(pred)),
                "r"(a), "r"(lo), "r"(hi)
                : "memory");
 }
@@ -197,7 +217,7 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
   const BandGeo<C> g(P, task, wsm);
   const int n = g.n;
   const int nch = (n + CH - 1) / CH;
-  const uint32_t from_c = g.hdr, to_c = g.hdr + (DO_REF ? 8 : 16);
+  const uint32_t from_c = g.hdr, to_ref = g.hdr + 8, to_st = g.hdr + 16;
   uint32_t wmask = 0;  // RAGGED: bit i = word 32i+t of the row segment exists
 #pragma unroll
   for (int i = 0; i < K; ++i) wmask |= static_cast<uint32_t>(32 * i + t < g.ws) << i;
@@ -206,29 +226,47 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
   const uint64_t gS0 = reinterpret_cast<uint64_t>(g.S + g.c0 + t);
   int consumed = 0, complete = 0;  // cached compute-warp progress
   int landed = 0, stored = 0;      // published to the compute warp
-  // chunk k of ref: rows CH*k+1 .. CH*k+CH (row i of the chunk: K copies per lane)
+  // chunk k of ref: rows CH*k+1 .. CH*k+CH (row i of the chunk: K copies per lane).  Chunks are
+  // issued / stored in order, so the global row pointers advance incrementally; ring offsets
+  // within a chunk are compile-time immediates (a chunk never wraps: RR, SR multiples of CH).
+  uint64_t gR = SEQ ? 0ull : gR0 + ldr4;  // (row CH*kr+1, word t) of the next ref chunk
   auto issue_chunk = [&](int k) {
     if constexpr (!SEQ) {
+      const uint32_t d0 = g.refR + static_cast<uint32_t>((CH * k) & (RR - 1)) * RS4 + 4u * t;
+      uint64_t gsrc = gR;
+      gR += CH * ldr4;
+      if (!RAGGED && CH * k + CH <= n) {
+        [&]<int... R>(std::integer_sequence<int, R...>) {
+          ((cp_row<R * 4 * C::RS, K>(d0, gsrc), gsrc += ldr4), ...);
+        }(std::make_integer_sequence<int, CH>{});
+      } else {
 #pragma unroll
-      for (int i = 0; i < CH; ++i) {
-        const int ri = CH * k + 1 + i;
-        const uint64_t gsrc = gR0 + static_cast<uint64_t>(static_cast<long long>(ri)) * ldr4;
-        const uint32_t d = g.refR + static_cast<uint32_t>((ri - 1) & (RR - 1)) * RS4 + 4u * t;
-        if (ri <= n) {
-          if constexpr (!RAGGED) {
-            [&]<int... I>(std::integer_sequence<int, I...>) { (cp_async4_imm<128 * I>(d, gsrc), ...); }(std::make_integer_sequence<int, K>{});
-          } else {
+        for (int i = 0; i < CH; ++i) {
+          const int ri = CH * k + 1 + i;
+          const uint32_t d = d0 + static_cast<uint32_t>(i) * RS4;
+          if (ri <= n) {
             [&]<int... I>(std::integer_sequence<int, I...>) {
-              (cp_async4_imm_p<128 * I>((wmask >> I) & 1u, d, gsrc), ...);
+              (cp_async4_imm_p<128 * I>(!RAGGED || ((wmask >> I) & 1u), d, gsrc), ...);
             }(std::make_integer_sequence<int, K>{});
           }
+          gsrc += ldr4;
         }
       }
     }
   };
+  // L2 prefetch of chunk k's rows: CH rows x NL 128-byte lines, lane t handles lines t, t+32, ...
+  // (P.dbg_skip bit 5: one cp.async.bulk.prefetch.L2 per row instead)
+  const uint32_t pf_bytes = static_cast<uint32_t>((4 * g.ws + 12 + 15) & ~15);
   auto prefetch_chunk = [&](int k) {
     if constexpr (!SEQ) {
-      // CH rows x NL lines, lane t handles lines t, t+32, ...
+      if (P.dbg_skip & 32u) {
+        const int rp = CH * k + 1 + t;
+        if (t < CH && rp <= n) {
+          const uint64_t ga = (reinterpret_cast<uint64_t>(g.Rf + g.c0) + static_cast<uint64_t>(static_cast<long long>(rp)) * ldr4) & ~15ull;
+          asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(ga), "r"(pf_bytes) : "memory");
+        }
+        return;
+      }
 #pragma unroll
       for (int f = t; f < CH * C::NL; f += 32) {
         const int i = f / C::NL, ln = f - (f / C::NL) * C::NL;
@@ -242,28 +280,35 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
   // store converts back, one IADD3 per value: S = S' - r p - (c0 + 32 I + t) p
   int colp[K];
 #pragma unroll
-  for (int I = 0; I < K; ++I) colp[I] = (g.c0 + 32 * I + t) * g.p;
+  for (int I = 0; I < K; ++I) colp[I] = -(g.c0 + 32 * I + t) * g.p;
+  uint64_t gS = gS0 + lds4;  // (row CH*ks+1, word t) of the next score chunk
   auto store_chunk = [&](int k) {
-    int v[CH][K];
+    const uint32_t a0 = g.scR + static_cast<uint32_t>((CH * k) & (SR - 1)) * RS4 + 4u * t;
+    uint64_t ga = gS;
+    gS += CH * lds4;
+    int rp = -(CH * k + 1) * g.p;
+    if (!RAGGED && CH * k + CH <= n) {
+      // the common case: K LDS + K IADD3 + K unpredicated coalesced STG per row
+      int v[CH][K];
+      [&]<int... R>(std::integer_sequence<int, R...>) { (lds_row<R * 4 * C::RS, K>(a0, v[R]), ...); }(std::make_integer_sequence<int, CH>{});
 #pragma unroll
-    for (int i = 0; i < CH; ++i) {
-      const int ro = CH * k + 1 + i;
-      const uint32_t a = g.scR + static_cast<uint32_t>((ro - 1) & (SR - 1)) * RS4 + 4u * t;
-      [&]<int... I>(std::integer_sequence<int, I...>) { ((v[i][I] = lds32_imm<128 * I>(a)), ...); }(std::make_integer_sequence<int, K>{});
-    }
+      for (int i = 0; i < CH; ++i) {
+        [&]<int... I>(std::integer_sequence<int, I...>) { (stg32_imm<128 * I>(ga, v[i][I] + rp + colp[I]), ...); }(std::make_integer_sequence<int, K>{});
+        ga += lds4;
+        rp -= g.p;
+      }
+    } else {
 #pragma unroll
-    for (int i = 0; i < CH; ++i) {
-      const int ro = CH * k + 1 + i;
-      const int rp = ro * g.p;
-#pragma unroll
-      for (int I = 0; I < K; ++I) v[i][I] = v[i][I] - rp - colp[I];
-      const uint64_t ga = gS0 + static_cast<uint64_t>(static_cast<long long>(ro)) * lds4;
-      if constexpr (!RAGGED) {
-        [&]<int... I>(std::integer_sequence<int, I...>) { (stg32_imm_p<128 * I>(ro <= n, ga, v[i][I]), ...); }(std::make_integer_sequence<int, K>{});
-      } else {
+      for (int i = 0; i < CH; ++i) {
+        const int ro = CH * k + 1 + i;
+        const uint32_t a = a0 + static_cast<uint32_t>(i) * RS4;
+        int v[K];
+        [&]<int... I>(std::integer_sequence<int, I...>) { ((v[I] = lds32_imm<128 * I>(a)), ...); }(std::make_integer_sequence<int, K>{});
         [&]<int... I>(std::integer_sequence<int, I...>) {
-          (stg32_imm_p<128 * I>(ro <= n && ((wmask >> I) & 1u), ga, v[i][I]), ...);
+          (stg32_imm_p<128 * I>(ro <= n && (!RAGGED || ((wmask >> I) & 1u)), ga, v[I] + rp + colp[I]), ...);
         }(std::make_integer_sequence<int, K>{});
+        ga += lds4;
+        rp -= g.p;
       }
     }
   };
@@ -302,6 +347,7 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
         did = true;
       }
     }
+    bool done = true;
     if constexpr (DO_REF) {
       int nl;
       if (SEQ || kr == nch) {
@@ -313,23 +359,30 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
       }
       if (nl > landed) {
         landed = nl;
-        prog_publish(to_c, landed, 0, (P.dbg_skip & 2u) != 0);  // __syncwarp: every lane's copies landed
+        prog_publish(to_ref, landed, 0, (P.dbg_skip & 2u) != 0);  // __syncwarp: every lane's copies landed
       }
-      if (landed == n) break;
-    } else {
+      done = landed == n;
+    }
+    if constexpr (DO_ST) {
       const int ns = min(n, CH * ks);
       if (ns > stored) {
         stored = ns;
-        prog_publish(to_c, stored, 0, (P.dbg_skip & 2u) != 0);
+        prog_publish(to_st, stored, 0, (P.dbg_skip & 2u) != 0);
       }
-      if (ks == nch) break;
+      done = done && ks == nch;
     }
+    if (done) break;
     if (did) {
       idle = 0;
-    } else if ((++idle & 255u) == 0) {
-      const uint64_t now = globaltimer_ns();
-      if (idle == 256) tw = now;
-      else if (now - tw > P.spin_limit_ns) watchdog_trap(P.err);
+    } else {
+      // idle: back off (a tight poll of the progress words competes with the compute warp's
+      // shared-memory / shuffle traffic in the SM's MIO pipe)
+      if (P.stage_sleep_ns) __nanosleep(P.stage_sleep_ns);
+      if ((++idle & 255u) == 0) {
+        const uint64_t now = globaltimer_ns();
+        if (idle == 256) tw = now;
+        else if (now - tw > P.spin_limit_ns) watchdog_trap(P.err);
+      }
     }
   }
   (void)tw0;
@@ -350,8 +403,9 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
   constexpr int BD = SRC == kSrcGlobal ? 1 : 3;  // border prefetch distance (blocks)
   const bool tracing = P.trace != nullptr;
   const unsigned long long t_task0 = tracing ? globaltimer_ns() : 0ull;
-  long long spin_cyc = 0, wait_cyc = 0, bp_cyc = 0;
-  const bool relaxed = (P.dbg_skip & 2u) != 0;
+  long long spin_cyc = 0, wait_cyc = 0, bp_cyc = 0, steady_cyc = 0, steady_blocks = 0;
+  long long ph_cyc[3] = {0, 0, 0}, st_wait_cyc = 0;  // event phases: publish + staging wait, border (+ spin), back-pressure + misc
+  const bool strict = (P.dbg_skip & 16u) != 0;  // (experiments: release-fenced progress stores)
 
   const BandGeo<C> g(P, task, wsm);
   const int n = g.n, p = g.p, band = g.band, c0 = g.c0, ws = g.ws;
@@ -568,8 +622,10 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
       }
       if constexpr (HALO_OUT) vo -= out_adj + s * p;
       st_entry_smem_p(do_out && sink_smem, bring_out + 8u * (r & (C::BR - 1)), static_cast<uint32_t>(vo), gen | static_cast<uint32_t>(r));
-      st_entry_gpu_p(do_out && sink_gpu, lout + r, static_cast<uint32_t>(vo), lout_tag);
-      st_entry_sys_p(do_out && sink_sys, lout + r, static_cast<uint32_t>(vo), lout_tag);
+      if constexpr (HALO_OUT)
+        st_entry_sys_p(do_out, lout + r, static_cast<uint32_t>(vo), lout_tag);
+      else
+        st_entry_gpu_p(do_out && sink_gpu, lout + r, static_cast<uint32_t>(vo), lout_tag);
     }
     vlast = Pv[K - 1];
   };
@@ -580,11 +636,16 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     const int sig0 = Q * CE;
     // ---- event Q.  To the staging warp: ref rows <= sig0-30 consumed (lane 31 read row sig0-30
     // at step sig0-1), score rows <= sig0-31 complete (lane 31 wrote row sig0-31 at step sig0-1).
-    prog_publish(to_s, max(0, sig0 - 30), max(0, sig0 - 31), relaxed);
+    const long long ce0 = tracing ? clock64() : 0;
+    // relaxed: the warp's earlier shared-memory accesses are performed in order before this
+    // store (__syncwarp, then one lane's store; the MIO processes a warp's shared-memory
+    // instructions in order) -- a release fence here cost ~200 cycles per event (MEMBAR.CTA)
+    prog_publish(to_s, max(0, sig0 - 30), max(0, sig0 - 31), !strict);
     {
       // this block reads ref rows <= sig0+CE+1 and rewrites score slots of rows <= sig0+CE
       const int need_l = SEQ ? 0 : min(n, sig0 + CE + 1), need_s = sig0 + CE - SR;
       if (landed < need_l || stored < need_s) {
+        const bool landed_short = !(landed < need_l);  // (trace) waiting on the store warp only
         const long long c0c = clock64();
         const uint64_t tw = globaltimer_ns();
         unsigned spins = 0;
@@ -596,8 +657,10 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
           if ((++spins & 255u) == 0 && globaltimer_ns() - tw > P.spin_limit_ns) watchdog_trap(P.err);
         }
         wait_cyc += clock64() - c0c;
+        if (landed_short) st_wait_cyc += clock64() - c0c;
       }
     }
+    const long long ce1 = tracing ? clock64() : 0;
     if constexpr (SRC == kSrcSmem) {
       cur = e1;
       if (sig0 + CE < nsteps) e1 = load_block(Q + 1);
@@ -628,6 +691,7 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     }
     curv = static_cast<int>(static_cast<uint32_t>(cur));
     if (conv_in) curv += (CE * Q + 1 + t) * p;
+    const long long ce2 = tracing ? clock64() : 0;
     if (sink_smem) {
       // rows written in this block are <= sig0+CE; the slot of row x held row x-BR
       const int need = sig0 + CE - C::BR;
@@ -643,13 +707,19 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     if constexpr (!SEQ) {
       if (Q == 0) load_ref_row(laneR + static_cast<uint32_t>((-t) & (RR - 1)) * RS4);  // row 1-t
     }
+    if (tracing) {
+      const long long ce3 = clock64();
+      ph_cyc[0] += ce1 - ce0, ph_cyc[1] += ce2 - ce1, ph_cyc[2] += ce3 - ce2;
+    }
     // ---- CE steps (two unrolled halves of CE/2)
     if (sig0 >= 31 && sig0 + CE <= n) {
+      const long long c0c = tracing ? clock64() : 0;
 #pragma unroll 1
       for (int h = 0; h < CE; h += CE / 2) {
 #pragma unroll
         for (int j = 0; j < CE / 2; ++j) step(sig0 + h + j, h + j, std::true_type{});
       }
+      if (tracing) steady_cyc += clock64() - c0c, ++steady_blocks;
     } else {
 #pragma unroll 1
       for (int h = 0; h < CE; h += CE / 2) {
@@ -658,7 +728,7 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
       }
     }
   }
-  prog_publish(to_s, n, n, relaxed);  // every row consumed and complete
+  prog_publish(to_s, n, n, !strict);  // every row consumed and complete
   if (tracing && t == 0 && task < P.trace_cap) {
     unsigned smid;
     asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
@@ -667,7 +737,10 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     e[1] = t_task0;
     e[2] = globaltimer_ns();
     e[3] = smid;
-    e[4] = 0;
+    e[4] = static_cast<unsigned long long>(steady_cyc) | (static_cast<unsigned long long>(steady_blocks) << 44);
+    if (P.trace2 != nullptr)
+      for (int k = 0; k < 3; ++k) P.trace2[8 * task + k] = static_cast<unsigned long long>(ph_cyc[k]);
+    if (P.trace2 != nullptr) P.trace2[8 * task + 3] = static_cast<unsigned long long>(st_wait_cyc);
     e[5] = static_cast<unsigned long long>(bp_cyc);
     e[6] = static_cast<unsigned long long>(spin_cyc);
     e[7] = static_cast<unsigned long long>(wait_cyc);
@@ -679,9 +752,11 @@ __global__ void __launch_bounds__(32 * C::NWARPS, 1) nw_wave_kernel(const __grid
   constexpr int NW = C::NW;
   extern __shared__ __align__(128) unsigned char smem[];
   const int t = threadIdx.x & 31;
-  const int wa = threadIdx.x >> 5;  // 0..NW-1 compute, NW..2NW-1 ref staging, 2NW..3NW-1 store staging
+  // warps 0..NW-1 compute; SPB = 1: NW..2NW-1 ref + store staging; SPB = 2: NW..2NW-1 ref,
+  // 2NW..3NW-1 store staging
+  const int wa = threadIdx.x >> 5;
   const bool staging = wa >= NW;
-  const int role = wa < NW ? 0 : (wa < 2 * NW ? kRoleRef : kRoleStore);
+  const int role = wa < NW ? 0 : (C::SPB == 1 ? (kRoleRef | kRoleStore) : (wa < 2 * NW ? kRoleRef : kRoleStore));
   const int w = wa % NW;  // the band slot this warp serves
   // CTA header: [0] group ticket, [8 + 4w] consumer progress of warp w, [128..] border rings
   unsigned long long* const s_group = reinterpret_cast<unsigned long long*>(smem);
@@ -708,7 +783,12 @@ __global__ void __launch_bounds__(32 * C::NWARPS, 1) nw_wave_kernel(const __grid
     if (task < P.ntasks) {
       const int band = static_cast<int>(task % P.nbands);
       const bool full = band_ws(P.width, band, C::W) == C::W;
-      if (role == kRoleRef) {
+      if (C::SPB == 1 && staging) {
+        if (full)
+          wave_stage<C, false, kRoleRef | kRoleStore>(P, task, t, wsm);
+        else
+          wave_stage<C, true, kRoleRef | kRoleStore>(P, task, t, wsm);
+      } else if (role == kRoleRef) {
         if (full)
           wave_stage<C, false, kRoleRef>(P, task, t, wsm);
         else

@@ -10,8 +10,14 @@ spin = t[:, 6] / ghz / 1e3
 wait = t[:, 7] / ghz / 1e3
 bp = t[:, 5] / ghz / 1e3
 steps = n + 31
+sc = (t[:, 4] & ((1 << 44) - 1)).astype(np.float64)
+sb = (t[:, 4] >> 44).astype(np.float64)
 print(f"bands={len(t)} span={(t[:, 2].max() - t0) / 1e3:.1f} us; band0 sweep {dur[0]:.1f} us "
       f"({(dur[0] - wait[0]) * 1e3 * ghz / steps:.1f} cyc/step excl. staging waits)")
 for k in sorted(set([0, 1, 2, len(t) // 2, len(t) - 1])):
     print(f"  band {k:4d}: start {(t[k, 1] - t0) / 1e3:8.1f} us sweep {dur[k]:8.1f} us spin {spin[k]:7.1f} us "
-          f"staging-wait {wait[k]:7.1f} us bp {bp[k]:6.1f} us  cyc/step(excl spin+wait) {(dur[k] - spin[k] - wait[k]) * 1e3 * ghz / steps:6.1f}")
+          f"staging-wait {wait[k]:7.1f} us bp {bp[k]:6.1f} us  cyc/step(excl spin+wait) {(dur[k] - spin[k] - wait[k]) * 1e3 * ghz / steps:6.1f}"
+          f" steady-block cyc/step {sc[k] / max(sb[k], 1) / 16:6.1f} ({int(sb[k])} blocks)")
+    if t.shape[1] >= 11:
+        nev = (n + 31 + 15) // 16
+        print(f"      per event cycles: publish+wait {t[k, 8] / nev:7.1f} (wait {t[k, 7] / nev:7.1f})  border {t[k, 9] / nev:7.1f} (spin {t[k, 6] / nev:7.1f})  bp+misc {t[k, 10] / nev:7.1f}  (wait on store warp only {t[k, 11] / nev:7.1f})")
