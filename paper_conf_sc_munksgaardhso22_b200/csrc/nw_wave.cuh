@@ -589,25 +589,18 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     if (!ALL) active = r >= 1 && r <= n;
     if (active) {
       // gap-normalised cell: S'(r,j) = max(S'(r-1,j-1) + ref'(r,j), S'(r-1,j), S'(r,j-1))
-      // x_m = max(diag + ref', up): one DPX each; the row's left chain is a plain prefix max
-      // (depth 4 with 3-input max) and the left value L enters with one max per cell.
+      // x_m = max(diag + ref', up); the row's left chain is a plain prefix max and the left
+      // value L enters with one max per cell.
       int x[K];
       x[0] = __viaddmax_s32(Lprev, rv[0], Pv[0]);
 #pragma unroll
       for (int m = 1; m < K; ++m) x[m] = __viaddmax_s32(Pv[m - 1], rv[m], Pv[m]);
+      // (written as a sequential chain: ptxas schedules it better than a hand-built max3 tree;
+      // scripts/ubench_sp.cu V=2 vs V=0: 80 vs 94 cycles per K = 8 step)
       int Y[K];
       Y[0] = x[0];
-      Y[1] = max(x[0], x[1]);
-      if constexpr (K >= 4) {
-        Y[2] = __vimax3_s32(x[0], x[1], x[2]);
-        Y[3] = __vimax3_s32(Y[1], x[2], x[3]);
-      }
-      if constexpr (K == 8) {
-        Y[4] = __vimax3_s32(Y[2], x[3], x[4]);
-        Y[5] = __vimax3_s32(Y[3], x[4], x[5]);
-        Y[6] = __vimax3_s32(Y[4], x[5], x[6]);
-        Y[7] = __vimax3_s32(Y[5], x[6], x[7]);
-      }
+#pragma unroll
+      for (int m = 1; m < K; ++m) Y[m] = max(Y[m - 1], x[m]);
 #pragma unroll
       for (int m = 0; m < K; ++m) Pv[m] = max(L, Y[m]);
       Lprev = L;

@@ -5,7 +5,7 @@
 #include <cstdio>
 #include <cuda_runtime.h>
 
-constexpr int NSTEP = 16384, R = 64;
+constexpr int NSTEP = 16384, R = 32;
 
 template <int K>
 __device__ __forceinline__ void ldsK(unsigned a, int* v) {
@@ -36,7 +36,10 @@ __device__ __forceinline__ int iaddfma(int a, int one, int b) {  // a * one + b:
 // V=0: x = max(d + (r + 2p), up) as the kernel writes it; V=1: r + 2p forced onto the FMA pipe
 // (IMAD) so x is one VIADDMNMX; V=2: like 1 with a sequential prefix (no 3-input max)
 template <int K, int V>
-__global__ void k_sp(int* out, long long* cyc, int p2, int one) {
+__global__ void k_sp(int* out, long long* cyc, int p2, int one, unsigned long long* gbuf) {
+  unsigned long long* gout = gbuf + static_cast<size_t>(blockIdx.x * 8 + (threadIdx.x >> 5)) * NSTEP;
+  const int tag = blockIdx.x + 1;
+  const int curv = threadIdx.x * 3 + p2;
   extern __shared__ __align__(16) int sm[];
   const int t = threadIdx.x & 31, w = threadIdx.x >> 5;
   constexpr int RS = 32 * K + 4;
@@ -54,12 +57,21 @@ __global__ void k_sp(int* out, long long* cyc, int p2, int one) {
   for (int s = 0; s < NSTEP; ++s) {
     int rv[K];
 #pragma unroll
-    for (int m = 0; m < K; ++m) rv[m] = V == 0 ? rvn[m] + p2 : iaddfma(rvn[m], one, p2);
+    for (int m = 0; m < K; ++m) rv[m] = (V == 1 || V == 3) ? iaddfma(rvn[m], one, p2) : rvn[m] + p2;
     ldsK<K>(laneR + ((s + 1) & (R - 1)) * 4u * RS, rvn);
-    const int from_left = __shfl_up_sync(0xffffffffu, vlast, 1);
-    const int L = t == 0 ? s : from_left;
+    int L;
+    if constexpr (V == 6 || V == 8) {
+      const int bval = __shfl_sync(0xffffffffu, curv, s & 15);
+      const int from_left = __shfl_up_sync(0xffffffffu, vlast, 1);
+      L = t == 0 ? bval : from_left;
+    } else if constexpr (V == 5) {
+      L = __shfl_sync(0xffffffffu, vlast, (t + 31) & 31);  // lane 31 carries the border value
+    } else {
+      const int from_left = __shfl_up_sync(0xffffffffu, vlast, 1);
+      L = t == 0 ? s : from_left;
+    }
     int x[K], Y[K];
-    if constexpr (V == 0) {
+    if constexpr (V != 1 && V != 3) {
       x[0] = __viaddmax_s32(Lprev, rv[0], Pv[0]);
 #pragma unroll
       for (int m = 1; m < K; ++m) x[m] = __viaddmax_s32(Pv[m - 1], rv[m], Pv[m]);
@@ -69,7 +81,7 @@ __global__ void k_sp(int* out, long long* cyc, int p2, int one) {
       for (int m = 1; m < K; ++m) x[m] = max(iaddfma(Pv[m - 1], one, rv[m]), Pv[m]);
     }
     Y[0] = x[0];
-    if constexpr (V == 2) {
+    if constexpr (V >= 2) {
 #pragma unroll
       for (int m = 1; m < K; ++m) Y[m] = max(Y[m - 1], x[m]);
     } else {
@@ -89,7 +101,15 @@ __global__ void k_sp(int* out, long long* cyc, int p2, int one) {
     for (int m = 0; m < K; ++m) Pv[m] = max(L, Y[m]);
     Lprev = L;
     stsK<K>(laneS + (s & (R - 1)) * 4u * RS, Pv);
+    if constexpr (V == 7 || V == 8) {
+      asm volatile("{ .reg .pred q; setp.ne.b32 q, %0, 0; @q st.relaxed.gpu.global.v2.b32 [%1], {%2, %3}; }" ::"r"(static_cast<int>(t == 31)),
+                   "l"(gout + s), "r"(Pv[K - 1]), "r"(tag)
+                   : "memory");
+    }
     vlast = Pv[K - 1];
+    if constexpr (V == 5) {
+      if (t == 31) vlast = s ^ rvn[0];  // (stand-in for the next row's border value)
+    }
   }
   long long t1 = clock64();
   int acc = 0;
@@ -105,10 +125,12 @@ void run(int nw, int sms) {
   long long* cyc;
   cudaMalloc(&out, sms * 32 * nw * 4);
   cudaMalloc(&cyc, sms * 32 * 8);
+  unsigned long long* gbuf;
+  cudaMalloc(&gbuf, static_cast<size_t>(sms) * 8 * NSTEP * 8);
   const int smem = nw * 2 * R * (32 * K + 4) * 4;
   cudaFuncSetAttribute(k_sp<K, V>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  k_sp<K, V><<<sms, 32 * nw, smem>>>(out, cyc, 20, 1);
-  k_sp<K, V><<<sms, 32 * nw, smem>>>(out, cyc, 20, 1);
+  k_sp<K, V><<<sms, 32 * nw, smem>>>(out, cyc, 20, 1, gbuf);
+  k_sp<K, V><<<sms, 32 * nw, smem>>>(out, cyc, 20, 1, gbuf);
   cudaError_t e = cudaDeviceSynchronize();
   long long h[32];
   cudaMemcpy(h, cyc, 32 * 8, cudaMemcpyDeviceToHost);
@@ -119,17 +141,19 @@ void run(int nw, int sms) {
          32.0 * K / cps, 32.0 * K * nw / cps, e == cudaSuccess ? "" : cudaGetErrorString(e));
   cudaFree(out);
   cudaFree(cyc);
+  cudaFree(gbuf);
 }
 
 int main() {
   int sms = 148;
-  for (int nw : {1, 2, 4, 8}) {
-    run<2, 1>(nw, sms);
-    run<4, 0>(nw, sms);
-    run<4, 1>(nw, sms);
-    run<8, 0>(nw, sms);
-    run<8, 1>(nw, sms);
+  for (int nw : {1}) {
     run<8, 2>(nw, sms);
+    run<8, 6>(nw, sms);
+    run<8, 7>(nw, sms);
+    run<8, 8>(nw, sms);
+    run<4, 0>(nw, sms);
+    run<4, 2>(nw, sms);
+    run<4, 8>(nw, sms);
   }
   return 0;
 }
