@@ -323,7 +323,7 @@ def main():
         torch.cuda.synchronize()
         nwb.nw_debug_set_trace(None)
         tt = tbuf.cpu().numpy()
-        np.save(args.trace, np.concatenate([tt[: 8 * ntask].reshape(ntask, 8), tt[8 * ntask:].reshape(ntask, 8)[:, :4]], 1))
+        np.save(args.trace, np.concatenate([tt[: 8 * ntask].reshape(ntask, 8), tt[8 * ntask:].reshape(ntask, 8)], 1))
     # ---- e2e through the public C ABI with host buffers (H2D + kernel + D2H inside the timing)
     if B == 1 and args.e2e_steps > 0 and args.variant == "strip" and not strips:
         hs = torch.empty((n + 1, n + 1), dtype=torch.int32, pin_memory=True)

@@ -73,8 +73,8 @@ nw_status check_range(int64_t n, int32_t p) {
 // v5 self-staging wavefront kernels (nw_wave.cuh)
 using WCfg8 = WaveCfg<8, false, 1, 2>;   // tile 0 / 256: W = 256, one band per CTA, ref + store warps
 using WCfg8S = WaveCfg<8, true, 1, 2>;
-using WCfg4 = WaveCfg<4, false, 2, 1>;   // tile 16 .. 128: W = 128, two bands per CTA
-using WCfg4S = WaveCfg<4, true, 2, 1>;
+using WCfg4 = WaveCfg<4, false, 2, 2>;   // tile 16 .. 128: W = 128, two bands per CTA
+using WCfg4S = WaveCfg<4, true, 2, 2>;
 
 struct DevInfo {
   bool init = false;

@@ -51,7 +51,7 @@ namespace nwb200 {
 
 // K columns per lane (band width W = 32 K), SEQ (ref generated from the sequences), NW bands
 // (compute warps) per CTA, SPB staging warps per band (1: one warp moves ref in and score out;
-// 2: separate ref and store warps).  Warp w runs on SM sub-partition w % 4: the compute warps
+// 2: separate ref and store warps; 3: a ref warp and two store warps taking alternate chunks).  Warp w runs on SM sub-partition w % 4: the compute warps
 // take sub-partitions 0..NW-1 and the staging warps the others (NW * (1 + SPB) <= 4).
 template <int K_, bool SEQ_, int NW_, int SPB_>
 struct WaveCfg {
@@ -79,7 +79,7 @@ struct WaveCfg {
   static_assert((RS * 4 / 16) % 8 == DELTA, "bank-group shift");
   static_assert(kWarpSmem % 32 == 0 && kCtaHdr % 32 == 0 && (HDR_BYTES + 4 * (REF_WORDS + SR * RS)) % 32 == 0,
                 "32-byte aligned rings (the profile's half-swap flips address bit 4)");
-  static_assert(NL <= 32 && NW <= 8 && (SPB == 1 || SPB == 2) && NWARPS <= 4, "geometry: one warp per sub-partition");
+  static_assert(NL <= 32 && NW <= 8 && SPB >= 1 && SPB <= 3 && NWARPS <= 8, "geometry");
   static_assert(RR % CH == 0 && (RR & (RR - 1)) == 0 && SR % CH == 0 && (SR & (SR - 1)) == 0 && RR >= 64 && SR >= 64,
                 "rings of whole chunks, powers of two, large enough for the staging schedule");
 };
@@ -208,8 +208,12 @@ __device__ __forceinline__ void prog_read(uint32_t a, int& lo, int& hi) {
 // The staging warp of a band: ref rows in (8-row chunks of 4-byte cp.async, paced by the ring
 // space the compute warp has released), score rows out (LDS.32 + coalesced STG.32 once the compute
 // warp has completed them), L2 prefetch ahead of the ref stream.
+// half (store roles): -1 = every score chunk, 0 / 1 = the even / odd chunks (SPB = 3).  A store
+// warp publishes, in its progress word (hdr + 16 + 8 half), the index of its next chunk: all of
+// its chunks below it are stored.
 template <class C, bool RAGGED, int ROLE>
-__device__ __forceinline__ void wave_stage(const StripParams& P, const long long task, const int t, unsigned char* const wsm) {
+__device__ __forceinline__ void wave_stage(const StripParams& P, const long long task, const int t, unsigned char* const wsm,
+                                           const int half = -1) {
   constexpr bool DO_REF = (ROLE & kRoleRef) != 0, DO_ST = (ROLE & kRoleStore) != 0;
   constexpr int K = C::K, CH = C::CH, RR = C::RR, SR = C::SR;
   constexpr uint32_t RS4 = 4u * C::RS;
@@ -217,12 +221,14 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
   const BandGeo<C> g(P, task, wsm);
   const int n = g.n;
   const int nch = (n + CH - 1) / CH;
-  const uint32_t from_c = g.hdr, to_ref = g.hdr + 8, to_st = g.hdr + 16;
+  const uint32_t from_c = g.hdr, to_ref = g.hdr + 8, to_st = g.hdr + 16 + 8 * (half > 0);
+  const int kstep = half >= 0 ? 2 : 1;  // score chunks handled: ks, ks + kstep, ...
   uint32_t wmask = 0;  // RAGGED: bit i = word 32i+t of the row segment exists
 #pragma unroll
   for (int i = 0; i < K; ++i) wmask |= static_cast<uint32_t>(32 * i + t < g.ws) << i;
   const uint64_t ldr4 = 4ull * static_cast<uint64_t>(P.ldr), lds4 = 4ull * static_cast<uint64_t>(P.lds);
   const uint64_t gR0 = SEQ ? 0ull : reinterpret_cast<uint64_t>(g.Rf + g.c0 + t);  // (row 0, word t) of the ref segment
+  const bool strict = (P.dbg_skip & 16u) != 0;  // (experiments: release-fenced progress stores)
   const uint64_t gS0 = reinterpret_cast<uint64_t>(g.S + g.c0 + t);
   int consumed = 0, complete = 0;  // cached compute-warp progress
   int landed = 0, stored = 0;      // published to the compute warp
@@ -281,21 +287,28 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
   int colp[K];
 #pragma unroll
   for (int I = 0; I < K; ++I) colp[I] = -(g.c0 + 32 * I + t) * g.p;
-  uint64_t gS = gS0 + lds4;  // (row CH*ks+1, word t) of the next score chunk
+  uint64_t gS = gS0 + lds4 + (half > 0 ? CH * lds4 : 0ull);  // (row CH*ks+1, word t) of the next score chunk
   auto store_chunk = [&](int k) {
     const uint32_t a0 = g.scR + static_cast<uint32_t>((CH * k) & (SR - 1)) * RS4 + 4u * t;
     uint64_t ga = gS;
-    gS += CH * lds4;
+    gS += static_cast<uint64_t>(kstep * CH) * lds4;
     int rp = -(CH * k + 1) * g.p;
     if (!RAGGED && CH * k + CH <= n) {
       // the common case: K LDS + K IADD3 + K unpredicated coalesced STG per row
       int v[CH][K];
       [&]<int... R>(std::integer_sequence<int, R...>) { (lds_row<R * 4 * C::RS, K>(a0, v[R]), ...); }(std::make_integer_sequence<int, CH>{});
+      // all conversions first, then the stores back to back (an IADD3 -> STG pair per value
+      // serialises on the ALU latency: measured 11 cycles per value)
 #pragma unroll
       for (int i = 0; i < CH; ++i) {
-        [&]<int... I>(std::integer_sequence<int, I...>) { (stg32_imm<128 * I>(ga, v[i][I] + rp + colp[I]), ...); }(std::make_integer_sequence<int, K>{});
-        ga += lds4;
+#pragma unroll
+        for (int I = 0; I < K; ++I) v[i][I] += rp + colp[I];
         rp -= g.p;
+      }
+#pragma unroll
+      for (int i = 0; i < CH; ++i) {
+        [&]<int... I>(std::integer_sequence<int, I...>) { (stg32_imm<128 * I>(ga, v[i][I]), ...); }(std::make_integer_sequence<int, K>{});
+        ga += lds4;
       }
     } else {
 #pragma unroll
@@ -321,7 +334,9 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
   // with RR = 128 the ref stream runs about RR/2 rows ahead, so both waits are satisfiable
   // (no deadlock) and normally already satisfied.
   constexpr int LAG = 3;
-  int kr = (SEQ || !DO_REF) ? nch : 0, ks = DO_ST ? 0 : nch;
+  const bool tracing = P.trace2 != nullptr && task < P.trace_cap;
+  long long st_busy = 0, st_gap_sum = 0, st_last = tracing ? clock64() : 0;  // (trace) store-warp cycles
+  int kr = (SEQ || !DO_REF) ? nch : 0, ks = DO_ST ? max(half, 0) : nch;
   const uint64_t tw0 = globaltimer_ns();
   uint64_t tw = tw0;
   unsigned idle = 0;
@@ -339,11 +354,13 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
       }
     }
     if (ks < nch) {
-      const int need = min(n, CH * ks + CH);
+      const int need = min(n, CH * ks + CH);  // (chunk ks complete)
       if (complete < need) prog_read(from_c, consumed, complete);
       if (complete >= need) {
+        const long long cs0 = tracing ? clock64() : 0;
         if (!(P.dbg_skip & 9u)) store_chunk(ks);
-        ++ks;
+        if (tracing) st_busy += clock64() - cs0, st_gap_sum += cs0 - st_last, st_last = clock64();
+        ks += kstep;
         did = true;
       }
     }
@@ -359,17 +376,22 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
       }
       if (nl > landed) {
         landed = nl;
-        prog_publish(to_ref, landed, 0, (P.dbg_skip & 2u) != 0);  // __syncwarp: every lane's copies landed
+        // relaxed (no MEMBAR): every lane's copies have completed (wait_group) before the
+        // __syncwarp and this store; a fence here would also wait for nothing useful
+        prog_publish(to_ref, landed, 0, !strict);
       }
       done = landed == n;
     }
     if constexpr (DO_ST) {
-      const int ns = min(n, CH * ks);
+      const int ns = min(ks, nch);  // my chunks below ns are stored
       if (ns > stored) {
         stored = ns;
-        prog_publish(to_st, stored, 0, (P.dbg_skip & 2u) != 0);
+        // relaxed: what the compute warp needs is that the ring slots were READ, and every STG
+        // above consumed its LDS result before this store issues (a release fence would wait
+        // for the global stores to be acknowledged: ~130 cycles of compute-warp stall per event)
+        prog_publish(to_st, stored, 0, !strict);
       }
-      done = done && ks == nch;
+      done = done && ks >= nch;
     }
     if (done) break;
     if (did) {
@@ -386,6 +408,12 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
     }
   }
   (void)tw0;
+  if constexpr (DO_ST) {
+    if (tracing && t == 0) {
+      P.trace2[8 * task + 4] = static_cast<unsigned long long>(st_busy);
+      P.trace2[8 * task + 5] = static_cast<unsigned long long>(st_gap_sum);
+    }
+  }
 }
 
 // The compute warp of a band: the wavefront sweep (no staging instructions in the step).
@@ -404,7 +432,7 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
   const bool tracing = P.trace != nullptr;
   const unsigned long long t_task0 = tracing ? globaltimer_ns() : 0ull;
   long long spin_cyc = 0, wait_cyc = 0, bp_cyc = 0, steady_cyc = 0, steady_blocks = 0;
-  long long ph_cyc[3] = {0, 0, 0}, st_wait_cyc = 0;  // event phases: publish + staging wait, border (+ spin), back-pressure + misc
+  long long ph_cyc[3] = {0, 0, 0}, st_wait_cyc = 0, pub_cyc = 0;  // event phases: publish + staging wait, border (+ spin), back-pressure + misc
   const bool strict = (P.dbg_skip & 16u) != 0;  // (experiments: release-fenced progress stores)
 
   const BandGeo<C> g(P, task, wsm);
@@ -540,6 +568,17 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
   for (int m = 0; m < K; ++m) rvn[m] = 0;
   int bp_cache = 0;            // last consumer progress read (back-pressure, shared sink)
   int landed = 0, stored = 0;  // cached staging-warp progress
+  // store warps publish chunk indices (SPB = 3: two warps, even / odd chunks): rows stored
+  auto read_stored = [&]() -> int {
+    int a, unused;
+    prog_read(from_t, a, unused);
+    if constexpr (C::SPB == 3) {
+      int b;
+      prog_read(from_t + 8, b, unused);
+      a = min(a, b);
+    }
+    return min(n, C::CH * a);
+  };
   uint64_t cur = 0ull;
   int curv = 0;  // lane j < CE: S' of the border entry of row CE*Q+1+j (the current block)
   // band 0's border (score column 0 or a strip halo) holds the true S: S'(r, 0) = S(r, 0) + r p
@@ -634,9 +673,17 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     // store (__syncwarp, then one lane's store; the MIO processes a warp's shared-memory
     // instructions in order) -- a release fence here cost ~200 cycles per event (MEMBAR.CTA)
     prog_publish(to_s, max(0, sig0 - 30), max(0, sig0 - 31), !strict);
+    if (tracing) pub_cyc += clock64() - ce0;
     {
       // this block reads ref rows <= sig0+CE+1 and rewrites score slots of rows <= sig0+CE
       const int need_l = SEQ ? 0 : min(n, sig0 + CE + 1), need_s = sig0 + CE - SR;
+      // one direct read of each stale progress word first (the staging warps normally run ahead:
+      // the timed spin below is the exception, and its timer reads are not free)
+      if (landed < need_l || stored < need_s) {
+        int unused;
+        if (landed < need_l) prog_read(from_r, landed, unused);
+        if (stored < need_s) stored = read_stored();
+      }
       if (landed < need_l || stored < need_s) {
         const bool landed_short = !(landed < need_l);  // (trace) waiting on the store warp only
         const long long c0c = clock64();
@@ -645,7 +692,7 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
         int unused;
         for (;;) {
           if (landed < need_l) prog_read(from_r, landed, unused);
-          if (stored < need_s) prog_read(from_t, stored, unused);
+          if (stored < need_s) stored = read_stored();
           if (landed >= need_l && stored >= need_s) break;
           if ((++spins & 255u) == 0 && globaltimer_ns() - tw > P.spin_limit_ns) watchdog_trap(P.err);
         }
@@ -734,6 +781,7 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     if (P.trace2 != nullptr)
       for (int k = 0; k < 3; ++k) P.trace2[8 * task + k] = static_cast<unsigned long long>(ph_cyc[k]);
     if (P.trace2 != nullptr) P.trace2[8 * task + 3] = static_cast<unsigned long long>(st_wait_cyc);
+    if (P.trace2 != nullptr) P.trace2[8 * task + 6] = static_cast<unsigned long long>(pub_cyc);
     e[5] = static_cast<unsigned long long>(bp_cyc);
     e[6] = static_cast<unsigned long long>(spin_cyc);
     e[7] = static_cast<unsigned long long>(wait_cyc);
@@ -750,6 +798,7 @@ __global__ void __launch_bounds__(32 * C::NWARPS, 1) nw_wave_kernel(const __grid
   const int wa = threadIdx.x >> 5;
   const bool staging = wa >= NW;
   const int role = wa < NW ? 0 : (C::SPB == 1 ? (kRoleRef | kRoleStore) : (wa < 2 * NW ? kRoleRef : kRoleStore));
+  const int half = C::SPB == 3 && wa >= 2 * NW ? (wa >= 3 * NW ? 1 : 0) : -1;  // SPB = 3: even / odd score chunks
   const int w = wa % NW;  // the band slot this warp serves
   // CTA header: [0] group ticket, [8 + 4w] consumer progress of warp w, [128..] border rings
   unsigned long long* const s_group = reinterpret_cast<unsigned long long*>(smem);
@@ -762,6 +811,7 @@ __global__ void __launch_bounds__(32 * C::NWARPS, 1) nw_wave_kernel(const __grid
     st_release_cta_v2(smem_u32(wsm), 0u, 0u);
     st_release_cta_v2(smem_u32(wsm) + 8, 0u, 0u);
     st_release_cta_v2(smem_u32(wsm) + 16, 0u, 0u);
+    st_release_cta_v2(smem_u32(wsm) + 24, C::SPB == 3 ? 1u : 0x3fffffffu, 0u);  // odd-chunk store warp: next chunk 1
   }
   __syncthreads();
 
@@ -788,9 +838,9 @@ __global__ void __launch_bounds__(32 * C::NWARPS, 1) nw_wave_kernel(const __grid
           wave_stage<C, true, kRoleRef>(P, task, t, wsm);
       } else if (role == kRoleStore) {
         if (full)
-          wave_stage<C, false, kRoleStore>(P, task, t, wsm);
+          wave_stage<C, false, kRoleStore>(P, task, t, wsm, half);
         else
-          wave_stage<C, true, kRoleStore>(P, task, t, wsm);
+          wave_stage<C, true, kRoleStore>(P, task, t, wsm, half);
       } else {
         const bool last_band = band == P.nbands - 1;
         int sink;
@@ -830,6 +880,7 @@ __global__ void __launch_bounds__(32 * C::NWARPS, 1) nw_wave_kernel(const __grid
       st_release_cta_v2(smem_u32(wsm), 0u, 0u);
       st_release_cta_v2(smem_u32(wsm) + 8, 0u, 0u);
       st_release_cta_v2(smem_u32(wsm) + 16, 0u, 0u);
+    st_release_cta_v2(smem_u32(wsm) + 24, C::SPB == 3 ? 1u : 0x3fffffffu, 0u);  // odd-chunk store warp: next chunk 1
     }
     __syncthreads();
     ++gcount;

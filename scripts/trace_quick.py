@@ -20,4 +20,7 @@ for k in sorted(set([0, 1, 2, len(t) // 2, len(t) - 1])):
           f" steady-block cyc/step {sc[k] / max(sb[k], 1) / 16:6.1f} ({int(sb[k])} blocks)")
     if t.shape[1] >= 11:
         nev = (n + 31 + 15) // 16
-        print(f"      per event cycles: publish+wait {t[k, 8] / nev:7.1f} (wait {t[k, 7] / nev:7.1f})  border {t[k, 9] / nev:7.1f} (spin {t[k, 6] / nev:7.1f})  bp+misc {t[k, 10] / nev:7.1f}  (wait on store warp only {t[k, 11] / nev:7.1f})")
+        if t.shape[1] >= 14:
+            nch = (n + 7) // 8
+            print(f"      store warp: busy {t[k, 12] / nch:7.1f} cyc/chunk, gap before chunk {t[k, 13] / nch:7.1f} cyc/chunk")
+        print(f"      per event cycles: publish+wait {t[k, 8] / nev:7.1f} (wait {t[k, 7] / nev:7.1f})  border {t[k, 9] / nev:7.1f} (spin {t[k, 6] / nev:7.1f})  bp+misc {t[k, 10] / nev:7.1f}  (wait on store warp only {t[k, 11] / nev:7.1f})  publish alone {t[k, 14] / nev:7.1f}")
