@@ -298,7 +298,8 @@ def main():
     roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
             "traffic": ncu_traffic(cfg["workload"], tile), "peak_source": peak_src,
             "algorithmic_bytes_per_launch": int(bpc * cells_local),
-            "kernel": ("nw_strip_kernel<%d,%s>" % (4 if tile in (0, 128) else 2, args.variant == "seq"))
+            "kernel": ("nw_wave_kernel<WaveCfg<K=%d, SEQ=%d>> (W = %d columns per band)"
+                       % (nwb.nw_band_width(tile) // 32, int(args.variant == "seq"), nwb.nw_band_width(tile)))
             if args.variant in ("strip", "seq")
             else f"nw_diag_kernel<{tile}> x{nwb.nw_launch_count(1, n, tile)} launches (+copies: unopt)",
             "kernel_ms_mean": kern_ms, "kernel_ms_median": statistics.median(per_launch)}
@@ -344,8 +345,42 @@ def main():
         out["gpu_launches_e2e"] = args.e2e_steps + 1
         nwb.nw_release_workspace()
         del hs, hr
-    elif B > 1:
-        out["e2e"] = None
+    elif B > 1 and args.e2e_steps > 0:
+        # batch: end to end through the public binding on a bounded sub-batch per rank (pinned
+        # host ref + borders -> device, nw_fill_batch, score matrices -> host, every step)
+        sb = min(nb, 32)
+        hr = torch.empty((sb, n + 1, n + 1), dtype=torch.int32, pin_memory=True)
+        hs = torch.empty((sb, n + 1, n + 1), dtype=torch.int32, pin_memory=True)
+        hr.copy_(R[:sb].cpu())
+        hs.copy_(S[:sb].cpu())
+        ds = torch.empty_like(S[:sb])
+        dr = torch.empty_like(R[:sb])
+        ho = torch.empty_like(hs).pin_memory()
+
+        def e2e_step():
+            dr.copy_(hr, non_blocking=True)
+            ds.copy_(hs, non_blocking=True)
+            nwb.nw_fill_batch(ds, dr, p, tile)
+            ho.copy_(ds, non_blocking=True)
+        e2e_step()
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        t = time.perf_counter()
+        for _ in range(args.e2e_steps):
+            e2e_step()
+        torch.cuda.synchronize()
+        e2e_s = (time.perf_counter() - t) / args.e2e_steps
+        if world > 1:
+            tt = torch.tensor([e2e_s], device=dev)
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+            e2e_s = float(tt.item())
+        out["e2e"] = {"value": world * sb * n * n / e2e_s / 1e9, "unit": "GCUPS",
+                      "h2d_bytes_per_step": world * 2 * 4 * sb * (n + 1) ** 2,
+                      "d2h_bytes_per_step": world * 4 * sb * (n + 1) ** 2, "ms_per_step": e2e_s * 1e3,
+                      "api": f"nw_fill_batch on a {sb}-pair sub-batch per rank (pinned host buffers)"}
+        out["gpu_launches_e2e"] = args.e2e_steps + 1
+        del hr, hs, ds, dr, ho
     gpu_last = S[n].cpu().numpy() if B == 1 and not strips else None
     if rank == 0 and not args.no_cpu:
         out["cpu_baseline"] = cpu_baseline(cfg, gpu_last)

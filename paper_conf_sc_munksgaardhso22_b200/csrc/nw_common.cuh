@@ -1,0 +1,133 @@
+// nw_common.cuh — definitions shared by the wavefront kernel (nw_wave.cuh) and the host side:
+// the band schedule (exported by nw_strip_map for pin P7), the kernel parameter block, the
+// border-source / sink kinds, small shared-memory / PTX helpers and the spin watchdog.
+//
+// What the path computes (Fig. 2, with Rodinia's cell function, R1):
+//     score[i][j] = max(score[i-1][j-1] + ref[i][j], score[i-1][j] - p, score[i][j-1] - p)
+// for every interior cell, each value written ONCE, in place (the short-circuited update of
+// P:512-516 / P:616-656: no temporary, no copy).
+#pragma once
+#include <cstdint>
+#include <type_traits>
+
+#include "nw_ptx.cuh"
+
+namespace nwb200 {
+
+constexpr unsigned kErrWatchdog = 0xBADB0001u;
+
+// ---- the schedule (shared by the kernel and the host export nw_strip_map, pin P7) --------
+// Band k of a pair covers columns [band_c0, band_c0 + band_ws); at wavefront step s lane t
+// computes row lane_row(s, t) (if 1 <= row <= n), columns band_c0 + t*K .. + K - 1 (clipped).
+__host__ __device__ __forceinline__ int band_c0(int band, int W) { return 1 + band * W; }
+__host__ __device__ __forceinline__ int band_ws(long long width, int band, int W) {
+  const long long r = width - static_cast<long long>(band) * W;
+  return static_cast<int>(r < W ? r : W);
+}
+__host__ __device__ __forceinline__ int lane_row(int step, int lane) { return step + 1 - lane; }
+// entries per band-border slot in the global border buffer: >= n+2 (16-byte pair reads may touch
+// row n+1) and even (every slot starts 16-byte aligned)
+__host__ __device__ __forceinline__ long long xstride(long long n) { return (n + 3) & ~1ll; }
+
+struct StripParams {
+  int32_t* score;
+  int64_t lds, pss;  // pitch, pair stride (elements)
+  const int32_t* ref;
+  int64_t ldr, psr;
+  int64_t n;       // rows 1..n
+  int64_t width;   // interior columns 1..width
+  int32_t p;
+  int32_t nbands;  // bands per pair
+  int64_t ntasks;  // pairs * nbands
+  int64_t ngroups; // ceil(ntasks / NW)
+  uint64_t* xbuf;  // [pairs][nbands-1][n+1] epoch-tagged right borders (inter-CTA handoffs)
+  uint32_t epoch;  // tag of this launch (xbuf)
+  const uint64_t* halo_in;  // left border of band 0 (sharded rank > 0) or null (use score col 0)
+  uint64_t* halo_out;       // right border of the last band (sharded, peer) or null
+  uint32_t halo_epoch;
+  int32_t halo_out_sys;
+  unsigned long long* ticket;
+  unsigned long long ticket_base;
+  unsigned int* err;
+  unsigned long long spin_limit_ns;
+  unsigned long long* trace;  // debug: per task 8 x u64 (see nw.h nw_debug_set_trace) or null
+  long long trace_cap;
+  unsigned long long* trace2;  // debug: per task {store cycles, ref-issue cycles} or null
+  unsigned int dbg_skip;       // timing experiments only (results invalid when nonzero)
+  unsigned int stage_sleep_ns; // staging-warp back-off when idle (NW_STAGE_SLEEP_NS, default below)
+  // NEXT-2 (SEQ kernels): ref[i][j] = subst[a[i-1]][b[j-1]] generated on chip
+  const uint8_t* seq_a;
+  const uint8_t* seq_b;
+  int64_t psa, psb;  // pair strides of a / b (bytes)
+  int8_t subst[32 * 32];
+};
+
+__device__ __forceinline__ int prmt_sext(uint32_t w, uint32_t sel) {
+  uint32_t d;
+  asm("prmt.b32 %0, %1, 0, %2;" : "=r"(d) : "r"(w), "r"(sel));
+  return static_cast<int>(d);
+}
+// opaque copy: keeps a value in a register (stops the compiler re-deriving smem bases per step)
+__device__ __forceinline__ uint32_t opaque(uint32_t x) {
+  asm volatile("mov.b32 %0, %0;" : "+r"(x));
+  return x;
+}
+// ref-ring load: not volatile (the compiler may hoist it inside a staging block for ILP), but it
+// consumes the token produced after the chunk's mbarrier wait, so it never moves above it
+__device__ __forceinline__ int lds_tok(uint32_t a, uint32_t tok) {
+  int v;
+  asm("ld.shared.b32 %0, [%1];" : "=r"(v) : "r"(a), "r"(tok));
+  return v;
+}
+__device__ __forceinline__ uint32_t mbar_wait_tok(uint32_t bar, uint32_t parity) {
+  mbar_wait(bar, parity);
+  uint32_t tk;
+  asm volatile("mov.u32 %0, 0;" : "=r"(tk)::"memory");
+  return tk;
+}
+__device__ __forceinline__ uint64_t lds64_volatile(uint32_t a) {
+  uint64_t v;
+  asm volatile("ld.volatile.shared.b64 %0, [%1];" : "=l"(v) : "r"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ int lds32_volatile(uint32_t a) {
+  int v;
+  asm volatile("ld.volatile.shared.b32 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ void sts32_volatile(uint32_t a, int v) {
+  asm volatile("st.volatile.shared.b32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+// predicated border-entry publishes (no branch in the step)
+__device__ __forceinline__ void st_entry_smem(bool pred, uint32_t a, uint32_t lo, uint32_t hi) {
+  asm volatile("{ .reg .pred q; .reg .b64 e; setp.ne.b32 q, %0, 0; mov.b64 e, {%2, %3}; @q st.volatile.shared.b64 [%1], e; }" ::"r"(
+                   static_cast<int>(pred)),
+               "r"(a), "r"(lo), "r"(hi)
+               : "memory");
+}
+__device__ __forceinline__ void st_entry_gpu(bool pred, uint64_t* p, uint32_t lo, uint32_t hi) {
+  asm volatile("{ .reg .pred q; .reg .b64 e; setp.ne.b32 q, %0, 0; mov.b64 e, {%2, %3}; @q st.relaxed.gpu.global.b64 [%1], e; }" ::"r"(
+                   static_cast<int>(pred)),
+               "l"(p), "r"(lo), "r"(hi)
+               : "memory");
+}
+__device__ __forceinline__ void st_entry_sys(bool pred, uint64_t* p, uint32_t lo, uint32_t hi) {
+  asm volatile("{ .reg .pred q; .reg .b64 e; setp.ne.b32 q, %0, 0; mov.b64 e, {%2, %3}; @q st.relaxed.sys.global.b64 [%1], e; }" ::"r"(
+                   static_cast<int>(pred)),
+               "l"(p), "r"(lo), "r"(hi)
+               : "memory");
+}
+
+__device__ __noinline__ void watchdog_trap(unsigned int* err) {
+  atomicExch(err, kErrWatchdog);
+  __trap();
+}
+
+// Border sources/sinks of one band (uniform per task)
+enum : int { kSrcPlain = 0, kSrcGlobal = 1, kSrcSmem = 2 };
+enum : int { kSinkNone = 0, kSinkSmem = 1, kSinkGlobal = 2 };
+
+// One band (task) of the persistent kernel; SINK is specialised so the steady-state step has no
+// branches.
+
+}  // namespace nwb200

@@ -2,7 +2,7 @@
 //
 // Synchronous validation, a per-(device, stream) workspace cache (ticket counter, epoch-tagged
 // band-border buffer, Unopt temporary), and the launches.  Every compute step runs in the
-// kernels of nw_strip.cuh / nw_diag.cuh; there is no CPU fallback: without a usable CUDA
+// kernels of nw_wave.cuh / nw_diag.cuh; there is no CPU fallback: without a usable CUDA
 // device the entry points return NW_ECUDA.
 #include <cuda_runtime.h>
 

@@ -6,7 +6,7 @@
 // for every interior cell, each value written ONCE, in place, into score (the short-circuited
 // update of P:512-516 / P:616-656: no temporary, no copy).
 //
-// Structure (same schedule as nw_strip.cuh, pinned by P7 through band_c0 / band_ws / lane_row):
+// Structure (the band schedule of nw_common.cuh, pinned by P7 through band_c0 / band_ws / lane_row):
 //   * A band = W = 32*K adjacent columns, all rows, swept by ONE warp; lane t owns the K adjacent
 //     columns c0+tK .. c0+tK+K-1 and at step s computes row s+1-t (the intra-tile anti-diagonals
 //     of P:498-501, skewed one row per lane).  The left value arrives from lane t-1 by SHFL.UP;
@@ -45,7 +45,7 @@
 #include <utility>
 
 #include "nw_ptx.cuh"
-#include "nw_strip.cuh"
+#include "nw_common.cuh"
 
 namespace nwb200 {
 
