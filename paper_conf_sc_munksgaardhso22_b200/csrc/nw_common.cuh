@@ -16,6 +16,14 @@ namespace nwb200 {
 
 constexpr unsigned kErrWatchdog = 0xBADB0001u;
 
+// Per-band timing instrumentation (nw_debug_set_trace / bench.py --trace) is compiled in only
+// with -DNW_TRACE=1 (NW_TRACE=1 python -m paper_conf_sc_munksgaardhso22_b200._build): its
+// runtime checks re-load the trace pointer from the constant bank at every event.
+#ifndef NW_TRACE
+#define NW_TRACE 0
+#endif
+constexpr bool kTrace = NW_TRACE != 0;
+
 // ---- the schedule (shared by the kernel and the host export nw_strip_map, pin P7) --------
 // Band k of a pair covers columns [band_c0, band_c0 + band_ws); at wavefront step s lane t
 // computes row lane_row(s, t) (if 1 <= row <= n), columns band_c0 + t*K .. + K - 1 (clipped).

@@ -334,7 +334,7 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
   // with RR = 128 the ref stream runs about RR/2 rows ahead, so both waits are satisfiable
   // (no deadlock) and normally already satisfied.
   constexpr int LAG = 3;
-  const bool tracing = P.trace2 != nullptr && task < P.trace_cap;
+  const bool tracing = kTrace && P.trace2 != nullptr && task < P.trace_cap;
   long long st_busy = 0, st_gap_sum = 0, st_last = tracing ? clock64() : 0;  // (trace) store-warp cycles
   int kr = (SEQ || !DO_REF) ? nch : 0, ks = DO_ST ? max(half, 0) : nch;
   const uint64_t tw0 = globaltimer_ns();
@@ -429,7 +429,7 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
   constexpr bool SEQ = C::SEQ;
   constexpr unsigned FULL = 0xffffffffu;
   constexpr int BD = SRC == kSrcGlobal ? 1 : 3;  // border prefetch distance (blocks)
-  const bool tracing = P.trace != nullptr;
+  const bool tracing = kTrace && P.trace != nullptr;
   const unsigned long long t_task0 = tracing ? globaltimer_ns() : 0ull;
   long long spin_cyc = 0, wait_cyc = 0, bp_cyc = 0, steady_cyc = 0, steady_blocks = 0;
   long long ph_cyc[3] = {0, 0, 0}, st_wait_cyc = 0, pub_cyc = 0;  // event phases: publish + staging wait, border (+ spin), back-pressure + misc
@@ -778,7 +778,7 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     e[2] = globaltimer_ns();
     e[3] = smid;
     e[4] = static_cast<unsigned long long>(steady_cyc) | (static_cast<unsigned long long>(steady_blocks) << 44);
-    if (P.trace2 != nullptr)
+    if (kTrace && P.trace2 != nullptr)
       for (int k = 0; k < 3; ++k) P.trace2[8 * task + k] = static_cast<unsigned long long>(ph_cyc[k]);
     if (P.trace2 != nullptr) P.trace2[8 * task + 3] = static_cast<unsigned long long>(st_wait_cyc);
     if (P.trace2 != nullptr) P.trace2[8 * task + 6] = static_cast<unsigned long long>(pub_cyc);
