@@ -62,7 +62,7 @@ def lib() -> ctypes.CDLL:
         if _lib is None:
             if not os.path.exists(LIB_PATH):
                 raise RuntimeError(f"{LIB_PATH} is missing: run __graft_entry__.build() first")
-            L = ctypes.CDLL(LIB_PATH)
+            L = ctypes.CDLL(os.environ.get("NW_LIB") or LIB_PATH)  # NW_LIB: experiment builds only
             vp = ctypes.c_void_p
             L.nw_status_str.argtypes = [ctypes.c_int]
             L.nw_status_str.restype = ctypes.c_char_p

@@ -59,5 +59,15 @@ def build(force: bool = False, verbose: bool = False) -> str:
     return LIB_PATH
 
 
+def build_variant(out_path: str, defines) -> str:
+    """Experiments only: the library with extra -D flags at out_path (loaded via NW_LIB)."""
+    cmd = [nvcc(), *NVCC_FLAGS, *[f"-D{d}" for d in defines], "-I", INCLUDE, "-I", CSRC,
+           *[os.path.join(CSRC, s) for s in SOURCES], "-o", out_path]
+    r = subprocess.run(cmd, capture_output=True, text=True)
+    if r.returncode != 0:
+        raise RuntimeError(f"nvcc failed ({r.returncode}):\n{r.stderr[-4000:]}")
+    return out_path
+
+
 if __name__ == "__main__":
     print(build(force=True, verbose=True))

@@ -23,6 +23,11 @@ constexpr unsigned kErrWatchdog = 0xBADB0001u;
 #define NW_TRACE 0
 #endif
 constexpr bool kTrace = NW_TRACE != 0;
+// full bands publish their border entries two rows per 16-byte store (NW_PAIRS=0: one per row)
+#ifndef NW_PAIRS
+#define NW_PAIRS 1
+#endif
+constexpr bool kPairs = NW_PAIRS != 0;
 
 // ---- the schedule (shared by the kernel and the host export nw_strip_map, pin P7) --------
 // Band k of a pair covers columns [band_c0, band_c0 + band_ws); at wavefront step s lane t

@@ -71,10 +71,16 @@ nw_status check_range(int64_t n, int32_t p) {
 // Kernel instances: K columns per lane, SEQ (ref generated from the sequences), NW warps
 // (bands) per CTA (DESIGN.md §4.3 sizes the rings).
 // v5 self-staging wavefront kernels (nw_wave.cuh)
-using WCfg8 = WaveCfg<8, false, 1, 2>;   // tile 0 / 256: W = 256, one band per CTA, ref + store warps
-using WCfg8S = WaveCfg<8, true, 1, 2>;
-using WCfg4 = WaveCfg<4, false, 2, 2>;   // tile 16 .. 128: W = 128, two bands per CTA
-using WCfg4S = WaveCfg<4, true, 2, 2>;
+#ifndef NW_K8_SPB
+#define NW_K8_SPB 3
+#endif
+#ifndef NW_K4_SPB
+#define NW_K4_SPB 2
+#endif
+using WCfg8 = WaveCfg<8, false, 1, NW_K8_SPB>;   // tile 0 / 256: W = 256, one band per CTA, ref + store warps
+using WCfg8S = WaveCfg<8, true, 1, NW_K8_SPB>;
+using WCfg4 = WaveCfg<4, false, 2, NW_K4_SPB>;   // tile 16 .. 128: W = 128, two bands per CTA
+using WCfg4S = WaveCfg<4, true, 2, NW_K4_SPB>;
 
 struct DevInfo {
   bool init = false;

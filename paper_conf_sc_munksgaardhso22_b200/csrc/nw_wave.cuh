@@ -160,6 +160,26 @@ __device__ __forceinline__ void st_entry_smem_p(bool pred, uint32_t a, uint32_t 
                : "memory");
 }
 
+// two consecutive border entries (rows 2k, 2k+1: 16-byte aligned) in one v4 store
+__device__ __forceinline__ void st_pair_gpu_p(bool pred, uint64_t* p, uint32_t v0, uint32_t t0, uint32_t v1, uint32_t t1) {
+  asm volatile("{ .reg .pred q; setp.ne.b32 q, %0, 0; @q st.relaxed.gpu.global.v4.b32 [%1], {%2, %3, %4, %5}; }" ::"r"(
+                   static_cast<int>(pred)),
+               "l"(p), "r"(v0), "r"(t0), "r"(v1), "r"(t1)
+               : "memory");
+}
+__device__ __forceinline__ void st_pair_sys_p(bool pred, uint64_t* p, uint32_t v0, uint32_t t0, uint32_t v1, uint32_t t1) {
+  asm volatile("{ .reg .pred q; setp.ne.b32 q, %0, 0; @q st.relaxed.sys.global.v4.b32 [%1], {%2, %3, %4, %5}; }" ::"r"(
+                   static_cast<int>(pred)),
+               "l"(p), "r"(v0), "r"(t0), "r"(v1), "r"(t1)
+               : "memory");
+}
+__device__ __forceinline__ void st_pair_smem_p(bool pred, uint32_t a, uint32_t v0, uint32_t t0, uint32_t v1, uint32_t t1) {
+  asm volatile("{ .reg .pred q; setp.ne.b32 q, %0, 0; @q st.volatile.shared.v4.b32 [%1], {%2, %3, %4, %5}; }" ::"r"(
+                   static_cast<int>(pred)),
+               "r"(a), "r"(v0), "r"(t0), "r"(v1), "r"(t1)
+               : "memory");
+}
+
 enum : int { kRoleRef = 1, kRoleStore = 2 };  // staging-warp roles
 
 // Shared per-band geometry of the compute and staging warps.
@@ -598,7 +618,8 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
 
   // one wavefront step s (entry jj of the block's border window); ALL = every lane's row is in
   // 1..n (no predicates)
-  auto step = [&](const int s, const int jj, auto all_tag) {
+  int vprev = 0;  // the out lane's previous row value (paired border-entry stores)
+  auto step = [&](const int s, const int jj, auto all_tag, auto par_tag) {
     constexpr bool ALL = decltype(all_tag)::value;
     const int r = s + 1 - t;  // this lane's row
     // ---- ref of this step's row (loaded last step) and the next row's loads
@@ -653,11 +674,35 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
         for (int m = 0; m < K - 1; ++m) vo = out_m == m ? Pv[m] : vo;
       }
       if constexpr (HALO_OUT) vo -= out_adj + s * p;
-      st_entry_smem_p(do_out && sink_smem, bring_out + 8u * (r & (C::BR - 1)), static_cast<uint32_t>(vo), gen | static_cast<uint32_t>(r));
-      if constexpr (HALO_OUT)
-        st_entry_sys_p(do_out, lout + r, static_cast<uint32_t>(vo), lout_tag);
-      else
-        st_entry_gpu_p(do_out && sink_gpu, lout + r, static_cast<uint32_t>(vo), lout_tag);
+      if constexpr (!RAGGED && kPairs) {
+        // full band: the out lane is lane 31, so its row r = s - 30 has the parity of J.  Odd
+        // rows publish the pair (r-1, r) in one 16-byte store; an even last row is flushed alone.
+        constexpr bool ODD = decltype(par_tag)::value != 0;
+        const uint32_t ur = static_cast<uint32_t>(r);
+        if constexpr (ODD) {
+          st_pair_smem_p(do_out && sink_smem, bring_out + 8u * ((r - 1) & (C::BR - 1)), static_cast<uint32_t>(vprev), gen | (ur - 1),
+                         static_cast<uint32_t>(vo), gen | ur);
+          if constexpr (HALO_OUT)
+            st_pair_sys_p(do_out, lout + (r - 1), static_cast<uint32_t>(vprev), lout_tag, static_cast<uint32_t>(vo), lout_tag);
+          else
+            st_pair_gpu_p(do_out && sink_gpu, lout + (r - 1), static_cast<uint32_t>(vprev), lout_tag, static_cast<uint32_t>(vo), lout_tag);
+        } else if constexpr (!ALL) {
+          const bool fl = do_out && r == n;
+          st_pair_smem_p(fl && sink_smem, bring_out + 8u * (r & (C::BR - 1)), static_cast<uint32_t>(vo), gen | ur, static_cast<uint32_t>(vo),
+                         gen | (ur + 1));
+          if constexpr (HALO_OUT)
+            st_pair_sys_p(fl, lout + r, static_cast<uint32_t>(vo), lout_tag, static_cast<uint32_t>(vo), lout_tag);
+          else
+            st_pair_gpu_p(fl && sink_gpu, lout + r, static_cast<uint32_t>(vo), lout_tag, static_cast<uint32_t>(vo), lout_tag);
+        }
+        vprev = vo;
+      } else {
+        st_entry_smem_p(do_out && sink_smem, bring_out + 8u * (r & (C::BR - 1)), static_cast<uint32_t>(vo), gen | static_cast<uint32_t>(r));
+        if constexpr (HALO_OUT)
+          st_entry_sys_p(do_out, lout + r, static_cast<uint32_t>(vo), lout_tag);
+        else
+          st_entry_gpu_p(do_out && sink_gpu, lout + r, static_cast<uint32_t>(vo), lout_tag);
+      }
     }
     vlast = Pv[K - 1];
   };
@@ -756,15 +801,17 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
       const long long c0c = tracing ? clock64() : 0;
 #pragma unroll 1
       for (int h = 0; h < CE; h += CE / 2) {
-#pragma unroll
-        for (int j = 0; j < CE / 2; ++j) step(sig0 + h + j, h + j, std::true_type{});
+        [&]<int... J>(std::integer_sequence<int, J...>) {
+          (step(sig0 + h + J, h + J, std::true_type{}, std::integral_constant<int, J & 1>{}), ...);
+        }(std::make_integer_sequence<int, CE / 2>{});
       }
       if (tracing) steady_cyc += clock64() - c0c, ++steady_blocks;
     } else {
 #pragma unroll 1
       for (int h = 0; h < CE; h += CE / 2) {
-#pragma unroll
-        for (int j = 0; j < CE / 2; ++j) step(sig0 + h + j, h + j, std::false_type{});
+        [&]<int... J>(std::integer_sequence<int, J...>) {
+          (step(sig0 + h + J, h + J, std::false_type{}, std::integral_constant<int, J & 1>{}), ...);
+        }(std::make_integer_sequence<int, CE / 2>{});
       }
     }
   }
