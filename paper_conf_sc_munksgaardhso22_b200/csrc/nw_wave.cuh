@@ -53,6 +53,9 @@ namespace nwb200 {
 // (compute warps) per CTA, SPB staging warps per band (1: one warp moves ref in and score out;
 // 2: separate ref and store warps; 3: a ref warp and two store warps taking alternate chunks).  Warp w runs on SM sub-partition w % 4: the compute warps
 // take sub-partitions 0..NW-1 and the staging warps the others (NW * (1 + SPB) <= 4).
+#ifndef NW_RR
+#define NW_RR 128
+#endif
 template <int K_, bool SEQ_, int NW_, int SPB_>
 struct WaveCfg {
   static constexpr int K = K_, NW = NW_, SPB = SPB_;
@@ -62,7 +65,7 @@ struct WaveCfg {
   static constexpr int CE = 16;                 // compute-warp event period (steps) = border block (rows)
   static constexpr int DELTA = K == 4 ? 2 : 1;  // 16-byte bank-group shift per ring row
   static constexpr int RS = W + 4 * DELTA;      // ring row stride (words)
-  static constexpr int RR = 128;                // ref ring rows (the staging warp's lookahead)
+  static constexpr int RR = NW_RR;               // ref ring rows (the staging warp's lookahead)
   static constexpr int SR = 64;                 // score ring rows
   static constexpr int PFC = 12;                // L2 prefetch distance (chunks of CH rows) of the staging warp
   static constexpr int BR = 256;                // shared border ring entries
