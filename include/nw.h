@@ -31,9 +31,10 @@
  *   - `tile` b in {0, 16, 32, 64, 128, 256} selects the width W of the tile-column band one
  *     warp owns (W = 32K, K columns per lane): b in {0, 256} -> W = 256 (K = 8, the default),
  *     b in {16, 32, 64, 128} -> W = 128 (K = 4; narrower b x b tiles are processed 128/b side
- *     by side, because a lane's K ref values are 16-byte shared loads).  A CTA owns 1 (K=8) or
- *     2 (K=4) consecutive bands, each swept by a compute warp with a ref-staging and a
- *     store-staging warp.  The result does not depend on it (R8).
+ *     by side, because a lane's K ref values are 16-byte shared loads).  A CTA owns one band
+ *     (b in {0, 256, 32, 64}: a compute warp, a ref-staging warp and two store warps) or two
+ *     consecutive bands (b in {16, 128}: two compute warps, a ref and a store warp each).
+ *     The result does not depend on it (R8).
  *   - Any n >= 0 is accepted (ragged last band: n need not be a multiple of b).
  *   - Validation is synchronous and happens before anything is enqueued.  Range contract:
  *     0 <= penalty and 2*n*penalty + n*NW_REF_MAX < 2^31 (else NW_ERANGE), |ref| <= NW_REF_MAX

@@ -35,20 +35,30 @@ nw_status cuda_fail(cudaError_t e) {
 
 constexpr int64_t kMaxN = (int64_t{1} << 30) - 64;
 
-// tile -> K (columns per lane) of the wavefront kernel: band width W = 32 K.  The default
-// (tile 0) is the W = 256 kernel (measured fastest at n = 32768: one band per CTA, its compute,
-// ref-staging and store-staging warps on three SM sub-partitions); the paper's b x b tiles
-// (16/32/64) and 128 map to the W = 128 kernel (two bands per CTA, one staging warp per band).
-int tile_to_k(int32_t tile) {
+// tile -> kernel variant (WaveCfg below).  Band width W = 32 K.
+//   variant 0 (tile 0 / 256): K = 8, W = 256, one band per CTA (compute, ref and two store
+//             warps on the four SM sub-partitions) -- measured fastest at n = 32768;
+//   variant 1 (tiles 16, 128): K = 4, W = 128, two bands per CTA (border between them through
+//             shared memory), ref + store warp per band;
+//   variant 2 (tiles 32, 64):  K = 4, W = 128, one band per CTA with a ref and two store warps
+//             -- twice the CTAs of variant 1, for n where W = 128 bands are too few to fill the
+//             GPU two per SM (n = 16384: 128 bands).
+// The paper's b x b tile does not exist here (a band is W columns x all rows); every tile value
+// gives the same matrix (tested).
+int tile_to_variant(int32_t tile) {
   switch (tile) {
     case 0:
-    case 256: return 8;
+    case 256: return 0;
     case 16:
+    case 128: return 1;
     case 32:
-    case 64:
-    case 128: return 4;
-    default: return 0;
+    case 64: return 2;
+    default: return -1;
   }
+}
+int tile_to_k(int32_t tile) {
+  const int v = tile_to_variant(tile);
+  return v < 0 ? 0 : (v == 0 ? 8 : 4);
 }
 
 bool aligned4(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 3) == 0; }
@@ -79,13 +89,15 @@ nw_status check_range(int64_t n, int32_t p) {
 #endif
 using WCfg8 = WaveCfg<8, false, 1, NW_K8_SPB>;   // tile 0 / 256: W = 256, one band per CTA, ref + store warps
 using WCfg8S = WaveCfg<8, true, 1, NW_K8_SPB>;
-using WCfg4 = WaveCfg<4, false, 2, NW_K4_SPB>;   // tile 16 .. 128: W = 128, two bands per CTA
+using WCfg4 = WaveCfg<4, false, 2, NW_K4_SPB>;   // tiles 16, 128: W = 128, two bands per CTA
 using WCfg4S = WaveCfg<4, true, 2, NW_K4_SPB>;
+using WCfg41 = WaveCfg<4, false, 1, 3>;          // tiles 32, 64: W = 128, one band per CTA
+using WCfg41S = WaveCfg<4, true, 1, 3>;
 
 struct DevInfo {
   bool init = false;
   int sms = 0;
-  int wocc[2][2] = {{0, 0}, {0, 0}};  // resident CTAs per SM [K==4][SEQ]
+  int wocc[3][2] = {{0, 0}, {0, 0}, {0, 0}};  // resident CTAs per SM [variant][SEQ]
 };
 
 template <class C>
@@ -111,6 +123,8 @@ nw_status dev_info(int dev, DevInfo** out) {
     NW_CU((setup_wave<WCfg8S>(&d.wocc[0][1])));
     NW_CU((setup_wave<WCfg4>(&d.wocc[1][0])));
     NW_CU((setup_wave<WCfg4S>(&d.wocc[1][1])));
+    NW_CU((setup_wave<WCfg41>(&d.wocc[2][0])));
+    NW_CU((setup_wave<WCfg41S>(&d.wocc[2][1])));
     for (auto& r : d.wocc)
       for (int o : r)
         if (o < 1) return cuda_fail(cudaErrorInvalidConfiguration);
@@ -210,7 +224,8 @@ nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* 
   P.p = p;
   P.nbands = static_cast<int32_t>(nbands);
   P.ntasks = pairs * nbands;
-  const int NW = K == 8 ? WCfg8::NW : WCfg4::NW;
+  const int var = tile_to_variant(tile);
+  const int NW = var == 0 ? WCfg8::NW : (var == 1 ? WCfg4::NW : WCfg41::NW);
   P.ngroups = (P.ntasks + NW - 1) / NW;
   P.xbuf = w->xbuf;
   P.epoch = ++w->epoch;
@@ -243,21 +258,25 @@ nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* 
     P.psb = psb;
     for (int i = 0; i < 32 * 32; ++i) P.subst[i] = subst32[i];
   }
-  const int occ = di->wocc[K == 4][SEQ];
+  const int occ = di->wocc[var][SEQ];
   int64_t grid = static_cast<int64_t>(occ) * di->sms;
   if (g_debug_grid > 0) grid = g_debug_grid;
   if (grid > P.ngroups) grid = P.ngroups;
   P.ticket_base = w->ticket_next;
   w->ticket_next += static_cast<unsigned long long>(P.ngroups + grid);  // every CTA draws one extra ticket
   const unsigned g = static_cast<unsigned>(grid);
-  if (K == 8 && !SEQ)
+  if (var == 0 && !SEQ)
     nw_wave_kernel<WCfg8><<<g, 32 * WCfg8::NWARPS, WCfg8::kSmem, st>>>(P);
-  else if (K == 8)
+  else if (var == 0)
     nw_wave_kernel<WCfg8S><<<g, 32 * WCfg8S::NWARPS, WCfg8S::kSmem, st>>>(P);
-  else if (!SEQ)
+  else if (var == 1 && !SEQ)
     nw_wave_kernel<WCfg4><<<g, 32 * WCfg4::NWARPS, WCfg4::kSmem, st>>>(P);
-  else
+  else if (var == 1)
     nw_wave_kernel<WCfg4S><<<g, 32 * WCfg4S::NWARPS, WCfg4S::kSmem, st>>>(P);
+  else if (!SEQ)
+    nw_wave_kernel<WCfg41><<<g, 32 * WCfg41::NWARPS, WCfg41::kSmem, st>>>(P);
+  else
+    nw_wave_kernel<WCfg41S><<<g, 32 * WCfg41S::NWARPS, WCfg41S::kSmem, st>>>(P);
   NW_CU(cudaGetLastError());
   return NW_OK;
 }
@@ -503,14 +522,15 @@ nw_status nw_kernel_info(int32_t tile, int32_t device, int64_t* smem_bytes, int3
                          int32_t* num_sms) {
   const int K = tile_to_k(tile);
   if (!K) return NW_EINVAL;
-  if (smem_bytes) *smem_bytes = static_cast<int64_t>(K == 8 ? WCfg8::kSmem : WCfg4::kSmem);
+  const int var = tile_to_variant(tile);
+  if (smem_bytes) *smem_bytes = static_cast<int64_t>(var == 0 ? WCfg8::kSmem : (var == 1 ? WCfg4::kSmem : WCfg41::kSmem));
   if (!ctas_per_sm && !num_sms) return NW_OK;
   NW_CU(cudaSetDevice(device));
   std::lock_guard<std::mutex> lk(g_mu);
   DevInfo* di = nullptr;
   nw_status s = dev_info(device, &di);
   if (s != NW_OK) return s;
-  if (ctas_per_sm) *ctas_per_sm = di->wocc[K == 4][0];
+  if (ctas_per_sm) *ctas_per_sm = di->wocc[var][0];
   if (num_sms) *num_sms = di->sms;
   return NW_OK;
 }

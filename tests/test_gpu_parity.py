@@ -45,7 +45,7 @@ def gpu_fill(score, ref, p, tile, fn=None, ld=None, offset=0):
 SIZES = [1, 2, 3, 15, 16, 17, 31, 32, 33, 63, 64, 65, 100, 127, 128, 129, 255, 256, 257, 1000, 1024]
 
 
-@pytest.mark.parametrize("tile", [0, 16])
+@pytest.mark.parametrize("tile", [0, 16, 64])
 @pytest.mark.parametrize("n", SIZES)
 def test_fill_sizes(n, tile):
     score, ref = inputs.make_problem(n, 10, seed=n)
@@ -192,7 +192,7 @@ def _stream_compare(s_dev, score_row0, ref, n, p, chunk=2048):
     st.close()
 
 
-@pytest.mark.parametrize("n,tile", [(16384, 128), (32768, 0)])
+@pytest.mark.parametrize("n,tile", [(16384, 128), (16384, 64), (32768, 0)])
 def test_full_size_configs_bit_exact(n, tile):
     """BASELINE.json configs 2/3 at full size, in the launch configuration bench.py times:
     every cell against the streaming oracle."""
@@ -208,7 +208,7 @@ def test_full_size_configs_bit_exact(n, tile):
     _stream_compare(s_dev, score[0], ref, n, p)
 
 
-@pytest.mark.parametrize("tile", [0, 128])
+@pytest.mark.parametrize("tile", [0, 64, 128])
 @pytest.mark.parametrize("n", [1, 5, 31, 64, 129, 1000, 4096])
 def test_fill_seq_next2(n, tile):
     """NEXT-2: ref generated on chip from (a, b, BLOSUM62) == nw_fill on the materialised ref."""
