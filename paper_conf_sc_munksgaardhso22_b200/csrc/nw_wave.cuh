@@ -578,8 +578,8 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
       for (int m = 0; m < K; ++m)
         prof[(x * 32 + t) * K + 4 * ((m >> 2) ^ sw) + (m & 3)] = static_cast<int>(P.subst[x * 32 + bj[m]]) + 2 * p;
     }
-    a_cur = A[min(max(-t, 0), n - 1)] & 31;     // row 1-t
-    a_nxt = A[min(max(1 - t, 0), n - 1)] & 31;  // row 2-t
+    a_cur = A[min(max(1 - t, 0), n - 1)] & 31;  // row 2-t (row 1-t's profile row is loaded at event 0)
+    a_nxt = A[min(max(2 - t, 0), n - 1)] & 31;  // row 3-t
     __syncwarp();
   }
   const uint32_t profA = opaque(g.prof + 4u * K * t + 16u * sw);
@@ -610,6 +610,15 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
   const int out_adj = HALO_OUT ? (c0 + ws - 1 + 1 - out_lane) * p : 0;  // + s p = (r + c_last) p at step s
   int vlast = Pv[K - 1];
   const uint32_t laneR = opaque(g.refR + 16u * (K / 4) * t), laneS = opaque(g.scR + 16u * (K / 4) * t);
+  auto load_prof_row = [&](int a) {  // SEQ: this lane's K profile values for residue a
+    const uint32_t a0 = profA + (static_cast<uint32_t>(a) << (7 + (K == 8 ? 3 : 2)));  // + a * 32 lanes * 4K bytes
+    const int4 u = lds128_tok<0>(a0, tok);
+    rvn[0] = u.x, rvn[1] = u.y, rvn[2] = u.z, rvn[3] = u.w;
+    if constexpr (K == 8) {
+      const int4 v = lds128_tok<0>(a0 ^ 16u, tok);
+      rvn[4] = v.x, rvn[5] = v.y, rvn[6] = v.z, rvn[7] = v.w;
+    }
+  };
   auto load_ref_row = [&](uint32_t a) {  // K/4 LDS.128 of this lane's K ref values
     const int4 u = lds128_tok<0>(a, tok);
     rvn[0] = u.x, rvn[1] = u.y, rvn[2] = u.z, rvn[3] = u.w;
@@ -628,15 +637,13 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     // ---- ref of this step's row (loaded last step) and the next row's loads
     int rv[K];
     if constexpr (SEQ) {
-      const uint32_t a0 = profA + (static_cast<uint32_t>(a_cur) << (7 + (K == 8 ? 3 : 2)));  // + a * 32 lanes * 4K bytes
-      const int4 u = lds128_tok<0>(a0, tok);
-      rv[0] = u.x, rv[1] = u.y, rv[2] = u.z, rv[3] = u.w;
-      if constexpr (K == 8) {
-        const int4 v = lds128_tok<0>(a0 ^ 16u, tok);
-        rv[4] = v.x, rv[5] = v.y, rv[6] = v.z, rv[7] = v.w;
-      }
+      // the profile row of row r was loaded last step; load row r+1's now (its residue was
+      // fetched two steps ago) and fetch row r+3's residue
+#pragma unroll
+      for (int m = 0; m < K; ++m) rv[m] = rvn[m];
+      load_prof_row(a_cur);
       a_cur = a_nxt;
-      a_nxt = __ldg(A + min(max(r + 1, 0), n - 1)) & 31;  // residue of row r+2
+      a_nxt = __ldg(A + min(max(r + 2, 0), n - 1)) & 31;  // residue of row r+3
     } else {
       // ref' = ref + 2p (the diagonal move of the gap-normalised recurrence); off the
       // recurrence's critical path (the row was loaded one step ahead)
@@ -794,6 +801,8 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     asm volatile("mov.u32 %0, 0;" : "=r"(tok)::"memory");  // the block's ref loads stay below
     if constexpr (!SEQ) {
       if (Q == 0) load_ref_row(laneR + static_cast<uint32_t>((-t) & (RR - 1)) * RS4);  // row 1-t
+    } else {
+      if (Q == 0) load_prof_row(A[min(max(-t, 0), n - 1)] & 31);  // row 1-t
     }
     if (tracing) {
       const long long ce3 = clock64();
