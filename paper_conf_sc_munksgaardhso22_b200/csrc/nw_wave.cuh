@@ -761,13 +761,16 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
       if (sig0 + CE < nsteps) e1 = load_block(Q + 1);
       if (t == 0) sts32_volatile(prog_in, sig0);  // rows <= sig0 consumed (block Q-1 validated)
     } else {
-      if (sig0 + CE * BD < nsteps) prefetch_block(Q + BD);
-      cp_async_commit();  // this event's border copy
-      if constexpr (BD == 1)
-        cp_async_wait<1>();  // every earlier group landed: block Q's border entries
+      // block Q's copy is in the prologue's group (Q < BD) or in the one committed at the half
+      // point of block Q-BD; the groups committed after it may still be in flight
+      const int newer = min(Q, BD - 1);
+      if (newer == 0)
+        cp_async_wait<0>();
+      else if (newer == 1)
+        cp_async_wait<1>();
       else
-        cp_async_wait<3>();  // the groups of events <= Q-3 landed
-      __syncwarp();          // landed by lanes 0..CE-1, visible to the warp
+        cp_async_wait<2>();
+      __syncwarp();  // landed by lanes 0..CE-1, visible to the warp
       cur = read_block(Q);
     }
     if constexpr (SRC != kSrcPlain) {
@@ -813,6 +816,14 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
       const long long c0c = tracing ? clock64() : 0;
 #pragma unroll 1
       for (int h = 0; h < CE; h += CE / 2) {
+        if constexpr (SRC != kSrcSmem) {
+          // the border copy of block Q + BD, issued half a block before the event that first
+          // needs it (a fresher snapshot of the producer's column: less band-to-band lag)
+          if (h != 0) {
+            if (sig0 + CE * BD < nsteps) prefetch_block(Q + BD);
+            cp_async_commit();
+          }
+        }
         [&]<int... J>(std::integer_sequence<int, J...>) {
           (step(sig0 + h + J, h + J, std::true_type{}, std::integral_constant<int, J & 1>{}), ...);
         }(std::make_integer_sequence<int, CE / 2>{});
@@ -821,6 +832,14 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     } else {
 #pragma unroll 1
       for (int h = 0; h < CE; h += CE / 2) {
+        if constexpr (SRC != kSrcSmem) {
+          // the border copy of block Q + BD, issued half a block before the event that first
+          // needs it (a fresher snapshot of the producer's column: less band-to-band lag)
+          if (h != 0) {
+            if (sig0 + CE * BD < nsteps) prefetch_block(Q + BD);
+            cp_async_commit();
+          }
+        }
         [&]<int... J>(std::integer_sequence<int, J...>) {
           (step(sig0 + h + J, h + J, std::false_type{}, std::integral_constant<int, J & 1>{}), ...);
         }(std::make_integer_sequence<int, CE / 2>{});
