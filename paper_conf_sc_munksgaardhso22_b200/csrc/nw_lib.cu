@@ -6,6 +6,7 @@
 // device the entry points return NW_ECUDA.
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <cstdint>
 #include <cstdlib>
 #include <map>
@@ -91,12 +92,17 @@ using WCfg8 = WaveCfg<8, false, 1, NW_K8_SPB>;   // tile 0 / 256: W = 256, one b
 using WCfg8S = WaveCfg<8, true, 1, NW_K8_SPB>;
 using WCfg4 = WaveCfg<4, false, 2, NW_K4_SPB>;   // tiles 16, 128: W = 128, two bands per CTA
 using WCfg4S = WaveCfg<4, true, 2, NW_K4_SPB>;
+#ifndef NW_CLUSTER
+#define NW_CLUSTER 4
+#endif
+using WCfg8C = WaveCfg<8, false, 1, NW_K8_SPB, NW_CLUSTER>;  // variant 0, one pair: clusters (DSMEM handoff)
 using WCfg41 = WaveCfg<4, false, 1, 3>;          // tiles 32, 64: W = 128, one band per CTA
 using WCfg41S = WaveCfg<4, true, 1, 3>;
 
 struct DevInfo {
   bool init = false;
   int sms = 0;
+  int clusters = 0;  // co-resident clusters of the WCfg8C kernel (0: clusters unusable)
   int wocc[3][2] = {{0, 0}, {0, 0}, {0, 0}};  // resident CTAs per SM [variant][SEQ]
 };
 
@@ -125,6 +131,24 @@ nw_status dev_info(int dev, DevInfo** out) {
     NW_CU((setup_wave<WCfg4S>(&d.wocc[1][1])));
     NW_CU((setup_wave<WCfg41>(&d.wocc[2][0])));
     NW_CU((setup_wave<WCfg41S>(&d.wocc[2][1])));
+    {
+      int occ_c = 0;
+      if (setup_wave<WCfg8C>(&occ_c) == cudaSuccess) {
+        cudaLaunchConfig_t cfg = {};
+        cfg.gridDim = dim3(static_cast<unsigned>(WCfg8C::CL * 16));
+        cfg.blockDim = dim3(32 * WCfg8C::NWARPS);
+        cfg.dynamicSmemBytes = WCfg8C::kSmem;
+        cudaLaunchAttribute at[1];
+        at[0].id = cudaLaunchAttributeClusterDimension;
+        at[0].val.clusterDim.x = WCfg8C::CL;
+        at[0].val.clusterDim.y = 1;
+        at[0].val.clusterDim.z = 1;
+        cfg.attrs = at;
+        cfg.numAttrs = 1;
+        if (cudaOccupancyMaxActiveClusters(&d.clusters, nw_wave_kernel<WCfg8C>, &cfg) != cudaSuccess) d.clusters = 0;
+      }
+      (void)cudaGetLastError();
+    }
     for (auto& r : d.wocc)
       for (int o : r)
         if (o < 1) return cuda_fail(cudaErrorInvalidConfiguration);
@@ -226,7 +250,15 @@ nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* 
   P.ntasks = pairs * nbands;
   const int var = tile_to_variant(tile);
   const int NW = var == 0 ? WCfg8::NW : (var == 1 ? WCfg4::NW : WCfg41::NW);
-  P.ngroups = (P.ntasks + NW - 1) / NW;
+  // opt-in (env NW_CLUSTER=1): one pair on the K = 8 kernel as clusters of CL CTAs that hand
+  // the border column over through DSMEM.  Measured slower than the global-memory handoff at
+  // n = 32768 (318 vs 337 GCUPS with CL = 4; CL = 8 clusters do not all fit co-resident).
+  static const bool cluster_env = [] {
+    const char* e = std::getenv("NW_CLUSTER");
+    return e && e[0] == '1';
+  }();
+  const bool use_cluster = var == 0 && !SEQ && pairs == 1 && cluster_env && di->clusters > 0 && g_debug_grid == 0;
+  P.ngroups = use_cluster ? (P.ntasks + WCfg8C::CL - 1) / WCfg8C::CL : (P.ntasks + NW - 1) / NW;
   P.xbuf = w->xbuf;
   P.epoch = ++w->epoch;
   P.halo_in = halo_in;
@@ -257,6 +289,25 @@ nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* 
     P.psa = psa;
     P.psb = psb;
     for (int i = 0; i < 32 * 32; ++i) P.subst[i] = subst32[i];
+  }
+  if (use_cluster) {
+    const int64_t ncl = std::min<int64_t>(di->clusters, P.ngroups);
+    P.ticket_base = w->ticket_next;
+    w->ticket_next += static_cast<unsigned long long>(P.ngroups + ncl);  // every cluster draws one extra ticket
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(static_cast<unsigned>(ncl * WCfg8C::CL));
+    cfg.blockDim = dim3(32 * WCfg8C::NWARPS);
+    cfg.dynamicSmemBytes = WCfg8C::kSmem;
+    cfg.stream = st;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = WCfg8C::CL;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    NW_CU(cudaLaunchKernelEx(&cfg, nw_wave_kernel<WCfg8C>, P));
+    return NW_OK;
   }
   const int occ = di->wocc[var][SEQ];
   int64_t grid = static_cast<int64_t>(occ) * di->sms;

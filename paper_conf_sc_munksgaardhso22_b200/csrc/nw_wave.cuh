@@ -56,9 +56,12 @@ namespace nwb200 {
 #ifndef NW_RR
 #define NW_RR 128
 #endif
-template <int K_, bool SEQ_, int NW_, int SPB_>
+// CL > 1: thread-block clusters of CL CTAs (one band each, NW = 1) take CL consecutive bands;
+// inside a cluster the border column goes straight into the next CTA's shared memory (DSMEM).
+template <int K_, bool SEQ_, int NW_, int SPB_, int CL_ = 1>
 struct WaveCfg {
-  static constexpr int K = K_, NW = NW_, SPB = SPB_;
+  static constexpr int K = K_, NW = NW_, SPB = SPB_, CL = CL_;
+  static_assert(CL == 1 || NW == 1, "clusters of single-band CTAs");
   static constexpr bool SEQ = SEQ_;
   static constexpr int W = 32 * K;
   static constexpr int CH = 8;                  // staging chunk (rows)
@@ -76,7 +79,9 @@ struct WaveCfg {
   static constexpr int HDR_BYTES = 128;                // progress words: [0] compute -> staging, [8] ref -> compute, [16] store -> compute
   static constexpr int NWARPS = NW * (1 + SPB);        // per band: a compute warp and SPB staging warps
   static constexpr size_t kWarpSmem = HDR_BYTES + 4ull * (REF_WORDS + SR * RS + PROF_WORDS) + BPRE_BYTES;
-  static constexpr size_t kCtaHdr = 128 + static_cast<size_t>(NW - 1) * BR * 8;
+  // CTA header: ticket, progress words, the border rings between consecutive bands (NW - 1
+  // between the warps of the CTA; CL > 1: one incoming ring written by the previous CTA)
+  static constexpr size_t kCtaHdr = 128 + static_cast<size_t>(CL > 1 ? 1 : NW - 1) * BR * 8;
   static constexpr size_t kSmem = kCtaHdr + NW * kWarpSmem;
   static_assert(K == 4 || K == 8, "K/4 LDS.128 per step");
   static_assert((RS * 4 / 16) % 8 == DELTA, "bank-group shift");
@@ -181,6 +186,38 @@ __device__ __forceinline__ void st_pair_smem_p(bool pred, uint32_t a, uint32_t v
                    static_cast<int>(pred)),
                "r"(a), "r"(v0), "r"(t0), "r"(v1), "r"(t1)
                : "memory");
+}
+
+// DSMEM (shared::cluster addresses from mapa): the next CTA's incoming ring / progress word
+__device__ __forceinline__ uint32_t mapa_u32(uint32_t a, uint32_t rank) {
+  uint32_t d;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(d) : "r"(a), "r"(rank));
+  return d;
+}
+__device__ __forceinline__ void st_pair_dsmem_p(bool pred, uint32_t a, uint32_t v0, uint32_t t0, uint32_t v1, uint32_t t1) {
+  asm volatile("{ .reg .pred q; setp.ne.b32 q, %0, 0; @q st.relaxed.cluster.shared::cluster.v4.b32 [%1], {%2, %3, %4, %5}; }" ::"r"(
+                   static_cast<int>(pred)),
+               "r"(a), "r"(v0), "r"(t0), "r"(v1), "r"(t1)
+               : "memory");
+}
+__device__ __forceinline__ void st_entry_dsmem_p(bool pred, uint32_t a, uint32_t lo, uint32_t hi) {
+  asm volatile("{ .reg .pred q; setp.ne.b32 q, %0, 0; @q st.relaxed.cluster.shared::cluster.v2.b32 [%1], {%2, %3}; }" ::"r"(
+                   static_cast<int>(pred)),
+               "r"(a), "r"(lo), "r"(hi)
+               : "memory");
+}
+__device__ __forceinline__ int ld_dsmem_b32(uint32_t a) {
+  int v;
+  asm volatile("ld.relaxed.cluster.shared::cluster.b32 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ uint32_t cluster_ctarank() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ void cluster_sync_all() {
+  asm volatile("barrier.cluster.arrive.release.aligned; barrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
 
 enum : int { kRoleRef = 1, kRoleStore = 2 };  // staging-warp roles
@@ -443,7 +480,7 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
 // SRC (compile time): where the band's left border column comes from.
 // HALO_OUT (compile time): the band pushes its last column into a strip halo, whose entries
 // hold the true S (nw.h), not the kernel's gap-normalised S'.
-template <class C, bool RAGGED, int SRC, bool HALO_OUT>
+template <class C, bool RAGGED, int SRC, bool HALO_OUT, bool REMOTE = false>
 __device__ __forceinline__ void wave_band(const StripParams& P, const long long task, const int w, const int t,
                                           unsigned char* const smem, unsigned char* const wsm, const uint32_t gen,
                                           const int sink) {
@@ -478,10 +515,16 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     lin = P.xbuf + (pair * (P.nbands - 1) + band - 1) * xstride(n);
     lin_epoch = P.epoch;
   }
-  const uint32_t bring_in = s_bring + (w - 1) * C::BR * 8;
-  const uint32_t bring_out = s_bring + w * C::BR * 8;
-  const uint32_t prog_in = s_prog + 4 * w;         // written by this warp (consumer of w-1)
-  const uint32_t prog_out = s_prog + 4 * (w + 1);  // read by this warp (producer for w+1)
+  // CL > 1 (NW = 1): the incoming ring at s_bring is written by the previous CTA of the cluster;
+  // REMOTE: this band's out-ring / consumer progress live in the next CTA (DSMEM addresses)
+  const uint32_t bring_in = C::CL > 1 ? s_bring : s_bring + (w - 1) * C::BR * 8;
+  const uint32_t prog_in = s_prog + 4 * w;  // written by this warp (consumer of the previous band)
+  uint32_t bring_out = s_bring + w * C::BR * 8, prog_out = s_prog + 4 * (w + 1);
+  if constexpr (REMOTE) {
+    const uint32_t nxt = cluster_ctarank() + 1;
+    bring_out = mapa_u32(s_bring, nxt);
+    prog_out = mapa_u32(s_prog, nxt);
+  }
   const int32_t* const colp = g.S + (c0 - 1);      // plain left border column
   // ---- sink (right)
   uint64_t* lout = nullptr;
@@ -690,16 +733,24 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
         constexpr bool ODD = decltype(par_tag)::value != 0;
         const uint32_t ur = static_cast<uint32_t>(r);
         if constexpr (ODD) {
-          st_pair_smem_p(do_out && sink_smem, bring_out + 8u * ((r - 1) & (C::BR - 1)), static_cast<uint32_t>(vprev), gen | (ur - 1),
-                         static_cast<uint32_t>(vo), gen | ur);
+          if constexpr (REMOTE)
+            st_pair_dsmem_p(do_out && sink_smem, bring_out + 8u * ((r - 1) & (C::BR - 1)), static_cast<uint32_t>(vprev), gen | (ur - 1),
+                            static_cast<uint32_t>(vo), gen | ur);
+          else
+            st_pair_smem_p(do_out && sink_smem, bring_out + 8u * ((r - 1) & (C::BR - 1)), static_cast<uint32_t>(vprev), gen | (ur - 1),
+                           static_cast<uint32_t>(vo), gen | ur);
           if constexpr (HALO_OUT)
             st_pair_sys_p(do_out, lout + (r - 1), static_cast<uint32_t>(vprev), lout_tag, static_cast<uint32_t>(vo), lout_tag);
           else
             st_pair_gpu_p(do_out && sink_gpu, lout + (r - 1), static_cast<uint32_t>(vprev), lout_tag, static_cast<uint32_t>(vo), lout_tag);
         } else if constexpr (!ALL) {
           const bool fl = do_out && r == n;
-          st_pair_smem_p(fl && sink_smem, bring_out + 8u * (r & (C::BR - 1)), static_cast<uint32_t>(vo), gen | ur, static_cast<uint32_t>(vo),
-                         gen | (ur + 1));
+          if constexpr (REMOTE)
+            st_pair_dsmem_p(fl && sink_smem, bring_out + 8u * (r & (C::BR - 1)), static_cast<uint32_t>(vo), gen | ur, static_cast<uint32_t>(vo),
+                            gen | (ur + 1));
+          else
+            st_pair_smem_p(fl && sink_smem, bring_out + 8u * (r & (C::BR - 1)), static_cast<uint32_t>(vo), gen | ur, static_cast<uint32_t>(vo),
+                           gen | (ur + 1));
           if constexpr (HALO_OUT)
             st_pair_sys_p(fl, lout + r, static_cast<uint32_t>(vo), lout_tag, static_cast<uint32_t>(vo), lout_tag);
           else
@@ -707,7 +758,10 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
         }
         vprev = vo;
       } else {
-        st_entry_smem_p(do_out && sink_smem, bring_out + 8u * (r & (C::BR - 1)), static_cast<uint32_t>(vo), gen | static_cast<uint32_t>(r));
+        if constexpr (REMOTE)
+          st_entry_dsmem_p(do_out && sink_smem, bring_out + 8u * (r & (C::BR - 1)), static_cast<uint32_t>(vo), gen | static_cast<uint32_t>(r));
+        else
+          st_entry_smem_p(do_out && sink_smem, bring_out + 8u * (r & (C::BR - 1)), static_cast<uint32_t>(vo), gen | static_cast<uint32_t>(r));
         if constexpr (HALO_OUT)
           st_entry_sys_p(do_out, lout + r, static_cast<uint32_t>(vo), lout_tag);
         else
@@ -793,10 +847,11 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     if (sink_smem) {
       // rows written in this block are <= sig0+CE; the slot of row x held row x-BR
       const int need = sig0 + CE - C::BR;
-      if (need > bp_cache && need > (bp_cache = lds32_volatile(prog_out))) {
+      auto read_bp = [&]() -> int { return REMOTE ? ld_dsmem_b32(prog_out) : lds32_volatile(prog_out); };
+      if (need > bp_cache && need > (bp_cache = read_bp())) {
         const long long c0c = clock64();
         const uint64_t tw = globaltimer_ns();
-        while (need > (bp_cache = lds32_volatile(prog_out)))
+        while (need > (bp_cache = read_bp()))
           if (globaltimer_ns() - tw > P.spin_limit_ns) watchdog_trap(P.err);
         bp_cyc += clock64() - c0c;
       }
@@ -883,7 +938,7 @@ __global__ void __launch_bounds__(32 * C::NWARPS, 1) nw_wave_kernel(const __grid
   const uint32_t s_prog = smem_u32(smem + 8);
   unsigned char* const wsm = smem + C::kCtaHdr + w * C::kWarpSmem;
   // shared border rings start invalid (tag 0xFFFFFFFF never equals gen | row, row < 2^30)
-  for (int i = threadIdx.x; i < (NW - 1) * C::BR; i += 32 * C::NWARPS) reinterpret_cast<unsigned long long*>(smem + 128)[i] = ~0ull;
+  for (int i = threadIdx.x; i < (C::CL > 1 ? 1 : NW - 1) * C::BR; i += 32 * C::NWARPS) reinterpret_cast<unsigned long long*>(smem + 128)[i] = ~0ull;
   if (threadIdx.x < NW) sts32_volatile(s_prog + 4 * threadIdx.x, 0);
   if (!staging && t == 0) {  // band progress words
     st_release_cta_v2(smem_u32(wsm), 0u, 0u);
@@ -894,12 +949,25 @@ __global__ void __launch_bounds__(32 * C::NWARPS, 1) nw_wave_kernel(const __grid
   __syncthreads();
 
   int gcount = 0;  // groups processed by this CTA (generation of the shared border tags)
+  const uint32_t crank = C::CL > 1 ? cluster_ctarank() : 0u;
+  if constexpr (C::CL > 1) cluster_sync_all();  // every CTA's rings initialised before any remote store
   for (;;) {
-    if (threadIdx.x == 0) *s_group = atomicAdd(P.ticket, 1ull);
-    __syncthreads();
-    const long long group = static_cast<long long>(*s_group - P.ticket_base);
+    long long group;
+    if constexpr (C::CL > 1) {
+      // one ticket per cluster (rank 0 draws it); the cluster takes CL consecutive bands
+      if (crank == 0 && threadIdx.x == 0) *s_group = atomicAdd(P.ticket, 1ull);
+      cluster_sync_all();
+      unsigned long long tk;
+      asm volatile("ld.relaxed.cluster.shared::cluster.b64 %0, [%1];" : "=l"(tk) : "r"(mapa_u32(smem_u32(s_group), 0)) : "memory");
+      cluster_sync_all();  // every CTA read the ticket before rank 0 may draw the next one
+      group = static_cast<long long>(tk - P.ticket_base);
+    } else {
+      if (threadIdx.x == 0) *s_group = atomicAdd(P.ticket, 1ull);
+      __syncthreads();
+      group = static_cast<long long>(*s_group - P.ticket_base);
+    }
     if (group >= P.ngroups) break;
-    const long long task = group * NW + w;
+    const long long task = C::CL > 1 ? group * C::CL + crank : group * NW + w;
     const uint32_t gen = static_cast<uint32_t>(gcount & 3) << 30;
     if (task < P.ntasks) {
       const int band = static_cast<int>(task % P.nbands);
@@ -921,14 +989,25 @@ __global__ void __launch_bounds__(32 * C::NWARPS, 1) nw_wave_kernel(const __grid
           wave_stage<C, true, kRoleStore>(P, task, t, wsm, half);
       } else {
         const bool last_band = band == P.nbands - 1;
+        // position of the band in its group: the previous / next band of the group is in this CTA
+        // (NW > 1: warps w -1 / w + 1) or, with clusters, in the previous / next CTA
+        const int jpos = C::CL > 1 ? static_cast<int>(crank) : w, jlast = C::CL > 1 ? C::CL - 1 : NW - 1;
         int sink;
         if (last_band)
           sink = P.halo_out ? kSinkGlobal : kSinkNone;
         else
-          sink = (w < NW - 1) ? kSinkSmem : kSinkGlobal;
-        const int src = band == 0 ? (P.halo_in ? kSrcGlobal : kSrcPlain) : (w > 0 ? kSrcSmem : kSrcGlobal);
+          sink = (jpos < jlast) ? kSinkSmem : kSinkGlobal;
+        const int src = band == 0 ? (P.halo_in ? kSrcGlobal : kSrcPlain) : (jpos > 0 ? kSrcSmem : kSrcGlobal);
         const bool halo_out = last_band && P.halo_out;  // validated: such a band is full width
-        if (halo_out) {
+        if (C::CL > 1 && sink == kSinkSmem) {
+          if (!full) __trap();  // (unreachable: only the last band of a pair can be ragged)
+          if (src == kSrcGlobal)
+            wave_band<C, false, kSrcGlobal, false, true>(P, task, w, t, smem, wsm, gen, sink);
+          else if (src == kSrcSmem)
+            wave_band<C, false, kSrcSmem, false, true>(P, task, w, t, smem, wsm, gen, sink);
+          else
+            wave_band<C, false, kSrcPlain, false, true>(P, task, w, t, smem, wsm, gen, sink);
+        } else if (halo_out) {
           if (src == kSrcGlobal)
             wave_band<C, false, kSrcGlobal, true>(P, task, w, t, smem, wsm, gen, sink);
           else if (src == kSrcSmem)

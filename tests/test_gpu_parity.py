@@ -6,11 +6,15 @@ oracle's int32 values exactly.  The interior is pre-filled with the sentinel 0x8
 unwritten cell fails too.  Inputs come from the seeded generator in inputs/ (no arithmetic of
 the method there); expected values only ever come from oracle/.
 """
+import os
+
 import numpy as np
 import pytest
 
 import inputs
 import oracle
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 torch = pytest.importorskip("torch")
 import paper_conf_sc_munksgaardhso22_b200 as nwb  # noqa: E402
@@ -263,3 +267,26 @@ def test_config4_shape_batch_bit_exact():
     with ThreadPoolExecutor(8) as ex:
         ok = list(ex.map(check, range(B)))
     assert all(ok), [k for k, v in enumerate(ok) if not v][:10]
+
+
+@pytest.mark.gpu
+def test_cluster_dsmem_handoff_opt_in():
+    """NW_CLUSTER=1 (opt-in): single pairs run as clusters of 4 CTAs whose border columns pass
+    through distributed shared memory; bit-exact against the oracle (subprocess: the switch is
+    read once per process)."""
+    import subprocess
+    import sys
+    code = r'''
+import sys; sys.path.insert(0, %r)
+import numpy as np, torch, inputs, oracle, paper_conf_sc_munksgaardhso22_b200 as nwb
+for n in (1, 255, 256, 1000, 1024, 3000):
+    s, r = inputs.make_problem(n, 10)
+    want = oracle.nw_ref(s.copy(), r, 10)
+    S = torch.from_numpy(s).cuda(); R = torch.from_numpy(r).cuda()
+    nwb.nw_fill(S, R, 10, 0); torch.cuda.synchronize()
+    assert np.array_equal(S.cpu().numpy(), want), n
+print("ok")
+''' % ROOT
+    env = dict(os.environ, NW_CLUSTER="1")
+    out = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=600)
+    assert out.returncode == 0 and "ok" in out.stdout, out.stderr[-2000:]
