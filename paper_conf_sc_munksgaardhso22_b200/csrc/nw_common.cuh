@@ -52,7 +52,8 @@ struct StripParams {
   int32_t p;
   int32_t nbands;  // bands per pair
   int64_t ntasks;  // pairs * nbands
-  int64_t ngroups; // ceil(ntasks / NW)
+  int64_t ngroups; // ceil(ntasks / NW) (pair mode: pairs)
+  int32_t pair_mode;  // 1: a ticket is a whole pair, its bands swept one after the other (NW = 1)
   uint64_t* xbuf;  // [pairs][nbands-1][n+1] epoch-tagged right borders (inter-CTA handoffs)
   uint32_t epoch;  // tag of this launch (xbuf)
   const uint64_t* halo_in;  // left border of band 0 (sharded rank > 0) or null (use score col 0)

@@ -259,6 +259,16 @@ nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* 
   }();
   const bool use_cluster = var == 0 && !SEQ && pairs == 1 && cluster_env && di->clusters > 0 && g_debug_grid == 0;
   P.ngroups = use_cluster ? (P.ntasks + WCfg8C::CL - 1) / WCfg8C::CL : (P.ntasks + NW - 1) / NW;
+  // many independent pairs on a one-band-per-CTA kernel: whole pairs per ticket (pair mode).
+  // NW_PAIR_MODE=0 disables, =2 forces it for any batch (tests)
+  static const int pair_env = [] {
+    const char* e = std::getenv("NW_PAIR_MODE");
+    return e ? static_cast<int>(std::strtol(e, nullptr, 10)) : 1;
+  }();
+  if (!use_cluster && NW == 1 && nbands > 1 && pair_env != 0 && (pair_env == 2 ? pairs > 1 : pairs >= 2LL * di->sms)) {
+    P.pair_mode = 1;
+    P.ngroups = pairs;
+  }
   P.xbuf = w->xbuf;
   P.epoch = ++w->epoch;
   P.halo_in = halo_in;

@@ -967,7 +967,12 @@ __global__ void __launch_bounds__(32 * C::NWARPS, 1) nw_wave_kernel(const __grid
       group = static_cast<long long>(*s_group - P.ticket_base);
     }
     if (group >= P.ngroups) break;
-    const long long task = C::CL > 1 ? group * C::CL + crank : group * NW + w;
+    // pair mode (many independent pairs, NW = 1): a ticket is a whole pair and the CTA sweeps its
+    // bands one after the other -- band k's border column is already complete when it starts
+    // (no band-to-band pipeline fill, no polling)
+    const int nsub = P.pair_mode ? P.nbands : 1;
+    for (int sub = 0; sub < nsub; ++sub) {
+    const long long task = P.pair_mode ? group * P.nbands + sub : (C::CL > 1 ? group * C::CL + crank : group * NW + w);
     const uint32_t gen = static_cast<uint32_t>(gcount & 3) << 30;
     if (task < P.ntasks) {
       const int band = static_cast<int>(task % P.nbands);
@@ -1041,6 +1046,7 @@ __global__ void __launch_bounds__(32 * C::NWARPS, 1) nw_wave_kernel(const __grid
     }
     __syncthreads();
     ++gcount;
+    }
   }
 }
 

@@ -290,3 +290,29 @@ print("ok")
     env = dict(os.environ, NW_CLUSTER="1")
     out = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=600)
     assert out.returncode == 0 and "ok" in out.stdout, out.stderr[-2000:]
+
+
+@pytest.mark.gpu
+def test_pair_mode_batches_forced():
+    """Pair mode (a CTA sweeps all bands of a pair in turn; automatic for large batches) forced
+    on small ragged batches with NW_PAIR_MODE=2, both one-band-per-CTA kernels (tiles 0, 64)."""
+    import subprocess
+    import sys
+    code = r'''
+import sys; sys.path.insert(0, %r)
+import numpy as np, torch, inputs, oracle, paper_conf_sc_munksgaardhso22_b200 as nwb
+for B, n, tile in ((3, 700, 0), (5, 257, 64), (2, 1024, 0), (4, 1500, 64), (3, 100, 0)):
+    ss, rs, want = [], [], []
+    for k in range(B):
+        s, r = inputs.make_problem(n, 10, seed=inputs.pair_seed(k))
+        ss.append(s); rs.append(r); want.append(oracle.nw_ref(s.copy(), r, 10))
+    S = torch.from_numpy(np.stack(ss)).cuda(); R = torch.from_numpy(np.stack(rs)).cuda()
+    nwb.nw_fill_batch(S, R, 10, tile); torch.cuda.synchronize()
+    got = S.cpu().numpy()
+    for k in range(B):
+        assert np.array_equal(got[k], want[k]), (B, n, tile, k)
+print("ok")
+''' % ROOT
+    env = dict(os.environ, NW_PAIR_MODE="2")
+    out = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=600)
+    assert out.returncode == 0 and "ok" in out.stdout, out.stderr[-2000:]
