@@ -241,7 +241,7 @@ struct BandGeo {
     ws = band_ws(P.width, band, C::W);
     S = P.score + pair * P.pss;
     Rf = C::SEQ ? nullptr : P.ref + pair * P.psr;
-    hdr = smem_u32(wsm);
+    hdr = opaque(smem_u32(wsm));  // kept in a register (else ptxas re-derives the shared window per use)
     refR = hdr + C::HDR_BYTES;
     scR = refR + 4u * C::REF_WORDS;
     prof = scR + 4u * C::SR * C::RS;
@@ -281,7 +281,7 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
   const BandGeo<C> g(P, task, wsm);
   const int n = g.n;
   const int nch = (n + CH - 1) / CH;
-  const uint32_t from_c = g.hdr, to_ref = g.hdr + 8, to_st = g.hdr + 16 + 8 * (half > 0);
+  const uint32_t from_c = g.hdr, to_ref = opaque(g.hdr + 8), to_st = opaque(g.hdr + 16 + 8 * (half > 0));
   const int kstep = half >= 0 ? 2 : 1;  // score chunks handled: ks, ks + kstep, ...
   uint32_t wmask = 0;  // RAGGED: bit i = word 32i+t of the row segment exists
 #pragma unroll
@@ -499,9 +499,9 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
   const int n = g.n, p = g.p, band = g.band, c0 = g.c0, ws = g.ws;
   const long long pair = g.pair;
   const long long lds = P.lds;
-  const uint32_t to_s = g.hdr, from_r = g.hdr + 8, from_t = g.hdr + 16;
-  const uint32_t s_prog = smem_u32(smem + 8);     // [4w]: rows consumed by warp w (shared source)
-  const uint32_t s_bring = smem_u32(smem + 128);  // [w * BR * 8]: ring warp w -> w+1
+  const uint32_t to_s = g.hdr, from_r = opaque(g.hdr + 8), from_t = opaque(g.hdr + 16);
+  const uint32_t s_prog = opaque(smem_u32(smem + 8));     // [4w]: rows consumed by warp w (shared source)
+  const uint32_t s_bring = opaque(smem_u32(smem + 128));  // [w * BR * 8]: ring warp w -> w+1
 
   // ---- border source (left)
   const uint64_t* lin = nullptr;
