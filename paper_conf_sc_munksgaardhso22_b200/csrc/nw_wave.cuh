@@ -56,6 +56,12 @@ namespace nwb200 {
 #ifndef NW_RR
 #define NW_RR 128
 #endif
+#ifndef NW_SUB
+#define NW_SUB 8
+#endif
+#ifndef NW_PF_AT
+#define NW_PF_AT 8
+#endif
 // CL > 1: thread-block clusters of CL CTAs (one band each, NW = 1) take CL consecutive bands;
 // inside a cluster the border column goes straight into the next CTA's shared memory (DSMEM).
 template <int K_, bool SEQ_, int NW_, int SPB_, int CL_ = 1>
@@ -771,6 +777,9 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     vlast = Pv[K - 1];
   };
 
+  constexpr int kSub = NW_SUB;    // steps per unrolled sub-block (a divisor of CE)
+  constexpr int kPfAt = NW_PF_AT;  // border copy issued this many steps into the block (a multiple of kSub)
+  static_assert(CE % kSub == 0 && kPfAt % kSub == 0 && kPfAt > 0 && kPfAt < CE, "sub-block geometry");
   const int nsteps = n + 31;  // compute steps 0 .. n+30
   const int nblk = (nsteps + CE - 1) / CE;
   for (int Q = 0; Q < nblk; ++Q) {
@@ -870,34 +879,36 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     if (sig0 >= 31 && sig0 + CE <= n) {
       const long long c0c = tracing ? clock64() : 0;
 #pragma unroll 1
-      for (int h = 0; h < CE; h += CE / 2) {
+      for (int h = 0; h < CE; h += kSub) {
         if constexpr (SRC != kSrcSmem) {
-          // the border copy of block Q + BD, issued half a block before the event that first
-          // needs it (a fresher snapshot of the producer's column: less band-to-band lag)
-          if (h != 0) {
+          // the border copy of block Q + BD, issued kPfAt steps into the block before the event
+          // that first needs it (a fresher snapshot of the producer's column: less band-to-band
+          // lag; later than the half point the L2 round trip is exposed at the event)
+          if (h == kPfAt) {
             if (sig0 + CE * BD < nsteps) prefetch_block(Q + BD);
             cp_async_commit();
           }
         }
         [&]<int... J>(std::integer_sequence<int, J...>) {
           (step(sig0 + h + J, h + J, std::true_type{}, std::integral_constant<int, J & 1>{}), ...);
-        }(std::make_integer_sequence<int, CE / 2>{});
+        }(std::make_integer_sequence<int, kSub>{});
       }
       if (tracing) steady_cyc += clock64() - c0c, ++steady_blocks;
     } else {
 #pragma unroll 1
-      for (int h = 0; h < CE; h += CE / 2) {
+      for (int h = 0; h < CE; h += kSub) {
         if constexpr (SRC != kSrcSmem) {
-          // the border copy of block Q + BD, issued half a block before the event that first
-          // needs it (a fresher snapshot of the producer's column: less band-to-band lag)
-          if (h != 0) {
+          // the border copy of block Q + BD, issued kPfAt steps into the block before the event
+          // that first needs it (a fresher snapshot of the producer's column: less band-to-band
+          // lag; later than the half point the L2 round trip is exposed at the event)
+          if (h == kPfAt) {
             if (sig0 + CE * BD < nsteps) prefetch_block(Q + BD);
             cp_async_commit();
           }
         }
         [&]<int... J>(std::integer_sequence<int, J...>) {
           (step(sig0 + h + J, h + J, std::false_type{}, std::integral_constant<int, J & 1>{}), ...);
-        }(std::make_integer_sequence<int, CE / 2>{});
+        }(std::make_integer_sequence<int, kSub>{});
       }
     }
   }
