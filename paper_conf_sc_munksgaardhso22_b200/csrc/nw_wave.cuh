@@ -56,6 +56,9 @@ namespace nwb200 {
 #ifndef NW_RR
 #define NW_RR 128
 #endif
+#ifndef NW_PFC
+#define NW_PFC 12
+#endif
 #ifndef NW_SUB
 #define NW_SUB 8
 #endif
@@ -76,7 +79,7 @@ struct WaveCfg {
   static constexpr int RS = W + 4 * DELTA;      // ring row stride (words)
   static constexpr int RR = NW_RR;               // ref ring rows (the staging warp's lookahead)
   static constexpr int SR = 64;                 // score ring rows
-  static constexpr int PFC = 12;                // L2 prefetch distance (chunks of CH rows) of the staging warp
+  static constexpr int PFC = NW_PFC;            // L2 prefetch distance (chunks of CH rows) of the staging warp
   static constexpr int BR = 256;                // shared border ring entries
   static constexpr int NL = (4 * W + 127) / 128 + 1;  // 128-byte lines touched by one row segment
   static constexpr int REF_WORDS = SEQ ? 0 : RR * RS;
