@@ -143,9 +143,11 @@ nw_status nw_fill_seq_batch(int32_t* score, int64_t ld_score, int64_t stride_sco
 
 /* ---- end to end from HOST memory (bench e2e) ---------------------------------------
  * Copies ref (rows 1..n) and the borders host->device, runs nw_fill, copies the full score
- * matrix device->host.  Host buffers: (n+1)x(n+1) int32, pitch n+1; pinned memory is
- * fastest.  Synchronous: returns when score_host holds the result.  Device buffers are
- * cached per device and freed by nw_release_workspace(). */
+ * matrix device->host.  Host buffers: (n+1)x(n+1) int32, pitch n+1.  Pinned (device-mapped)
+ * buffers take the zero-copy path: the kernel reads ref and writes score over the host link
+ * directly, both directions overlapped with the wavefront (NW_HOST_ZEROCOPY=0 disables);
+ * pageable buffers are staged through cached device buffers.  Synchronous: returns when
+ * score_host holds the result.  Device buffers are freed by nw_release_workspace(). */
 nw_status nw_fill_host(int32_t* score_host, const int32_t* ref_host, int64_t n, int32_t penalty,
                        int32_t tile, int32_t device);
 

@@ -514,6 +514,31 @@ nw_status nw_fill_host(int32_t* score_host, const int32_t* ref_host, int64_t n, 
   NW_CU(cudaSetDevice(device));
   HostBufs& hb = g_host[device];
   const size_t elems = static_cast<size_t>(n + 1) * static_cast<size_t>(n + 1);
+  // Pinned (device-mapped) host buffers: the kernel streams ref in and score out over the host
+  // link itself (zero copy, both directions at once, overlapped with the wavefront) instead of
+  // copy-in / compute / copy-out.  Pageable buffers take the staged path below.
+  static const bool zero_copy = [] {
+    const char* e = std::getenv("NW_HOST_ZEROCOPY");
+    return !(e && e[0] == '0');
+  }();
+  if (zero_copy) {
+    cudaPointerAttributes as{}, ar{};
+    const bool ok = cudaPointerGetAttributes(&as, score_host) == cudaSuccess &&
+                    cudaPointerGetAttributes(&ar, ref_host) == cudaSuccess && as.type == cudaMemoryTypeHost &&
+                    ar.type == cudaMemoryTypeHost && as.devicePointer && ar.devicePointer;
+    (void)cudaGetLastError();
+    if (ok) {
+      {
+        std::lock_guard<std::mutex> lk(g_mu);
+        if (!hb.st) NW_CU(cudaStreamCreateWithFlags(&hb.st, cudaStreamNonBlocking));
+      }
+      s = launch_strip(static_cast<int32_t*>(as.devicePointer), n + 1, 0, static_cast<const int32_t*>(ar.devicePointer), n + 1, 0, 1, n,
+                       n, penalty, tile, nullptr, nullptr, 0, 0, hb.st);
+      if (s != NW_OK) return s;
+      NW_CU(cudaStreamSynchronize(hb.st));
+      return NW_OK;
+    }
+  }
   {
     std::lock_guard<std::mutex> lk(g_mu);
     if (!hb.st) NW_CU(cudaStreamCreateWithFlags(&hb.st, cudaStreamNonBlocking));

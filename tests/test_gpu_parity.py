@@ -126,6 +126,17 @@ def test_fill_host_e2e():
     np.testing.assert_array_equal(got, want)
 
 
+@pytest.mark.parametrize("n,tile", [(999, 0), (1500, 64), (3000, 0)])
+def test_fill_host_pinned_zero_copy(n, tile):
+    """Pinned host buffers: the kernel reads ref and writes score over the host link directly."""
+    score, ref = inputs.make_problem(n, 10, seed=23)
+    want = expect(score, ref, 10)
+    hs = torch.from_numpy(score.copy()).pin_memory()
+    hr = torch.from_numpy(ref).pin_memory()
+    nwb.nw_fill_host(hs.numpy(), hr.numpy(), 10, tile, 0)
+    np.testing.assert_array_equal(hs.numpy(), want)
+
+
 @pytest.mark.parametrize("B,n,tile", [(1, 64, 0), (5, 100, 16), (7, 257, 0), (33, 64, 64), (3, 2048, 0), (4, 700, 128)])
 def test_batch(B, n, tile):
     probs = [inputs.make_problem(n, 10, seed=inputs.pair_seed(k)) for k in range(B)]
