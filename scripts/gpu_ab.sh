@@ -6,5 +6,5 @@ timeout 600 python -m pytest tests/test_gpu_parity.py -q -x -k "fill_sizes or sh
 for tl in ${@:-0 128}; do
   timeout 300 python bench.py --steps 5 --warmup 3 --no-cpu --e2e-steps 0 --tile $tl --trace gpurun_out/trace_t$tl.npy > gpurun_out/bench_t$tl.json 2> gpurun_out/bench_t$tl.err; echo "tile $tl rc=$?"
   python -c "import json;j=json.loads(open('gpurun_out/bench_t$tl.json').read().splitlines()[-1]);print('tile $tl:',round(j['value'],1),'GCUPS',round(j['ms_per_step'],3),'ms frac',round(j['roofline']['frac'],3))"
-  python scripts/trace_analysis.py gpurun_out/trace_t$tl.npy 32768 | tail -6
+  python scripts/trace_quick.py gpurun_out/trace_t$tl.npy 32768 | tail -6
 done
