@@ -150,6 +150,10 @@ nw_status nw_fill_seq_batch(int32_t* score, int64_t ld_score, int64_t stride_sco
  * score_host holds the result.  Device buffers are freed by nw_release_workspace(). */
 nw_status nw_fill_host(int32_t* score_host, const int32_t* ref_host, int64_t n, int32_t penalty,
                        int32_t tile, int32_t device);
+/* nw_fill_batch_host: the same for `batch` independent pairs stored back to back
+ * ([batch][n+1][n+1] int32 host arrays, pair stride (n+1)^2), one launch (nw_fill_batch). */
+nw_status nw_fill_batch_host(int32_t* score_host, const int32_t* ref_host, int64_t batch, int64_t n,
+                             int32_t penalty, int32_t tile, int32_t device);
 
 /* ---- the paper's / Rodinia's structure, kept as baselines ----------------------------
  * nw_fill_diagonal: one kernel launch per tile anti-diagonal d = 0..2q-2 (q = ceil(n/b)),

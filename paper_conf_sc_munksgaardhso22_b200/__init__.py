@@ -21,7 +21,7 @@ import threading
 from ._build import LIB_PATH, build  # noqa: F401  (build() is re-exported for __graft_entry__)
 
 __all__ = [
-    "NwError", "lib", "nw_fill", "nw_fill_batch", "nw_fill_seq", "nw_fill_seq_batch", "nw_fill_sharded", "nw_fill_host",
+    "NwError", "lib", "nw_fill", "nw_fill_batch", "nw_fill_seq", "nw_fill_seq_batch", "nw_fill_sharded", "nw_fill_host", "nw_fill_batch_host",
     "nw_fill_diagonal", "nw_fill_unopt", "nw_band_width", "nw_launch_count", "nw_diag_lmad",
     "nw_kernel_info", "nw_strip_map", "nw_debug_set_grid", "nw_debug_set_trace", "nw_release_workspace", "nw_status_str",
 ]
@@ -76,6 +76,7 @@ def lib() -> ctypes.CDLL:
             L.nw_fill_seq.argtypes = [vp, _i64, vp, vp, _i64, vp, _i32, _i32, _i32, vp]
             L.nw_fill_seq_batch.argtypes = [vp, _i64, _i64, vp, vp, _i64, _i64, _i64, vp, _i32, _i32, _i32, vp]
             L.nw_fill_host.argtypes = [vp, vp, _i64, _i32, _i32, _i32]
+            L.nw_fill_batch_host.argtypes = [vp, vp, _i64, _i64, _i32, _i32, _i32]
             L.nw_fill_diagonal.argtypes = [vp, _i64, vp, _i64, _i64, _i32, _i32, vp]
             L.nw_fill_unopt.argtypes = [vp, _i64, vp, _i64, _i64, _i32, _i32, vp]
             L.nw_band_width.argtypes = [_i32]
@@ -94,7 +95,7 @@ def lib() -> ctypes.CDLL:
             L.nw_debug_set_grid.restype = None
             L.nw_release_workspace.restype = None
             for f in ("nw_fill", "nw_fill_ld", "nw_fill_batch", "nw_fill_batch_ld", "nw_fill_sharded",
-                      "nw_fill_host", "nw_fill_diagonal", "nw_fill_unopt", "nw_kernel_info", "nw_fill_seq",
+                      "nw_fill_host", "nw_fill_batch_host", "nw_fill_diagonal", "nw_fill_unopt", "nw_kernel_info", "nw_fill_seq",
                       "nw_fill_seq_batch"):
                 getattr(L, f).restype = ctypes.c_int
             _lib = L
@@ -245,6 +246,21 @@ def nw_fill_host(score, ref, penalty: int, tile: int = 0, device: int = 0):
         raise ValueError("host arrays must be (n+1, n+1)")
     _check(lib().nw_fill_host(score.ctypes.data, ref.ctypes.data, n, int(penalty), int(tile),
                               int(device)), "nw_fill_host")
+    return score
+
+
+def nw_fill_batch_host(score, ref, penalty: int, tile: int = 0, device: int = 0):
+    """End-to-end from host numpy arrays ((B, n+1, n+1) int32, C-contiguous); synchronous.
+    Pinned (e.g. torch pin_memory) arrays take the zero-copy path."""
+    import numpy as np
+    if score.dtype != np.int32 or ref.dtype != np.int32 or not score.flags.c_contiguous \
+            or not ref.flags.c_contiguous:
+        raise ValueError("host arrays must be C-contiguous int32")
+    if score.ndim != 3 or score.shape != ref.shape or score.shape[1] != score.shape[2]:
+        raise ValueError("host arrays must be (B, n+1, n+1)")
+    B, n = score.shape[0], score.shape[1] - 1
+    _check(lib().nw_fill_batch_host(score.ctypes.data, ref.ctypes.data, B, n, int(penalty), int(tile),
+                                    int(device)), "nw_fill_batch_host")
     return score
 
 

@@ -505,15 +505,20 @@ nw_status nw_fill_seq(int32_t* score, int64_t ld_score, const uint8_t* a, const 
   return nw_fill_seq_batch(score, ld_score, 0, a, b, 0, 1, n, subst, alphabet, penalty, tile, stream);
 }
 
-nw_status nw_fill_host(int32_t* score_host, const int32_t* ref_host, int64_t n, int32_t penalty, int32_t tile,
-                       int32_t device) {
-  if (!score_host || !ref_host || n < 0 || n > kMaxN || tile_to_k(tile) == 0) return NW_EINVAL;
+nw_status nw_fill_batch_host(int32_t* score_host, const int32_t* ref_host, int64_t batch, int64_t n, int32_t penalty,
+                             int32_t tile, int32_t device) {
+  if (!score_host || !ref_host || batch < 0 || n < 0 || n > kMaxN || tile_to_k(tile) == 0) return NW_EINVAL;
   if (device < 0 || device >= 128) return NW_EINVAL;
   nw_status s = check_range(n, penalty);
-  if (s != NW_OK || n == 0) return s;
+  if (s != NW_OK || n == 0 || batch == 0) return s;
   NW_CU(cudaSetDevice(device));
   HostBufs& hb = g_host[device];
-  const size_t elems = static_cast<size_t>(n + 1) * static_cast<size_t>(n + 1);
+  const size_t pair_elems = static_cast<size_t>(n + 1) * static_cast<size_t>(n + 1);
+  const size_t elems = pair_elems * static_cast<size_t>(batch);
+  {
+    std::lock_guard<std::mutex> lk(g_mu);
+    if (!hb.st) NW_CU(cudaStreamCreateWithFlags(&hb.st, cudaStreamNonBlocking));
+  }
   // Pinned (device-mapped) host buffers: the kernel streams ref in and score out over the host
   // link itself (zero copy, both directions at once, overlapped with the wavefront) instead of
   // copy-in / compute / copy-out.  Pageable buffers take the staged path below.
@@ -528,12 +533,9 @@ nw_status nw_fill_host(int32_t* score_host, const int32_t* ref_host, int64_t n, 
                     ar.type == cudaMemoryTypeHost && as.devicePointer && ar.devicePointer;
     (void)cudaGetLastError();
     if (ok) {
-      {
-        std::lock_guard<std::mutex> lk(g_mu);
-        if (!hb.st) NW_CU(cudaStreamCreateWithFlags(&hb.st, cudaStreamNonBlocking));
-      }
-      s = launch_strip(static_cast<int32_t*>(as.devicePointer), n + 1, 0, static_cast<const int32_t*>(ar.devicePointer), n + 1, 0, 1, n,
-                       n, penalty, tile, nullptr, nullptr, 0, 0, hb.st);
+      s = launch_strip(static_cast<int32_t*>(as.devicePointer), n + 1, static_cast<int64_t>(pair_elems),
+                       static_cast<const int32_t*>(ar.devicePointer), n + 1, static_cast<int64_t>(pair_elems), batch, n, n,
+                       penalty, tile, nullptr, nullptr, 0, 0, hb.st);
       if (s != NW_OK) return s;
       NW_CU(cudaStreamSynchronize(hb.st));
       return NW_OK;
@@ -541,7 +543,6 @@ nw_status nw_fill_host(int32_t* score_host, const int32_t* ref_host, int64_t n, 
   }
   {
     std::lock_guard<std::mutex> lk(g_mu);
-    if (!hb.st) NW_CU(cudaStreamCreateWithFlags(&hb.st, cudaStreamNonBlocking));
     if (elems > hb.elems) {
       if (hb.score) NW_CU(cudaFree(hb.score));
       if (hb.ref) NW_CU(cudaFree(hb.ref));
@@ -554,14 +555,23 @@ nw_status nw_fill_host(int32_t* score_host, const int32_t* ref_host, int64_t n, 
   }
   const size_t pitch = static_cast<size_t>(n + 1) * 4;
   NW_CU(cudaMemcpyAsync(hb.ref, ref_host, elems * 4, cudaMemcpyHostToDevice, hb.st));
-  NW_CU(cudaMemcpyAsync(hb.score, score_host, pitch, cudaMemcpyHostToDevice, hb.st));  // row 0
-  NW_CU(cudaMemcpy2DAsync(hb.score + (n + 1), pitch, score_host + (n + 1), pitch, 4, static_cast<size_t>(n),
-                          cudaMemcpyHostToDevice, hb.st));  // column 0, rows 1..n
-  s = launch_strip(hb.score, n + 1, 0, hb.ref, n + 1, 0, 1, n, n, penalty, tile, nullptr, nullptr, 0, 0, hb.st);
+  for (int64_t k = 0; k < batch; ++k) {  // borders only: row 0 and column 0 of each pair
+    int32_t* d = hb.score + k * static_cast<int64_t>(pair_elems);
+    const int32_t* h = score_host + k * static_cast<int64_t>(pair_elems);
+    NW_CU(cudaMemcpyAsync(d, h, pitch, cudaMemcpyHostToDevice, hb.st));
+    NW_CU(cudaMemcpy2DAsync(d + (n + 1), pitch, h + (n + 1), pitch, 4, static_cast<size_t>(n), cudaMemcpyHostToDevice, hb.st));
+  }
+  s = launch_strip(hb.score, n + 1, static_cast<int64_t>(pair_elems), hb.ref, n + 1, static_cast<int64_t>(pair_elems), batch, n, n,
+                   penalty, tile, nullptr, nullptr, 0, 0, hb.st);
   if (s != NW_OK) return s;
   NW_CU(cudaMemcpyAsync(score_host, hb.score, elems * 4, cudaMemcpyDeviceToHost, hb.st));
   NW_CU(cudaStreamSynchronize(hb.st));
   return NW_OK;
+}
+
+nw_status nw_fill_host(int32_t* score_host, const int32_t* ref_host, int64_t n, int32_t penalty, int32_t tile,
+                       int32_t device) {
+  return nw_fill_batch_host(score_host, ref_host, 1, n, penalty, tile, device);
 }
 
 nw_status nw_fill_diagonal(int32_t* score, int64_t ld_score, const int32_t* ref, int64_t ld_ref, int64_t n,

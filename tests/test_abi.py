@@ -113,6 +113,7 @@ def test_batch_and_sharded_validation(L):
 
 def test_host_entry_validation(L):
     assert L.nw_fill_host(None, None, 8, 10, 0, 0) == NW_EINVAL
+    assert L.nw_fill_batch_host(None, None, 2, 8, 10, 0, 0) == NW_EINVAL
     assert L.nw_fill_diagonal(FAKE_S, 65, FAKE_R, 65, 64, 10, 128, None) == NW_EINVAL  # diag: b <= 64
 
 

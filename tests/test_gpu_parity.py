@@ -137,6 +137,23 @@ def test_fill_host_pinned_zero_copy(n, tile):
     np.testing.assert_array_equal(hs.numpy(), want)
 
 
+@pytest.mark.parametrize("pinned", [False, True])
+def test_fill_batch_host(pinned):
+    """Batched end to end from host arrays: staged (pageable) and zero-copy (pinned)."""
+    B, n = 5, 300
+    ss, rs, want = [], [], []
+    for k in range(B):
+        s, r = inputs.make_problem(n, 10, seed=inputs.pair_seed(k))
+        ss.append(s); rs.append(r); want.append(expect(s, r, 10))
+    S, R = np.stack(ss), np.stack(rs)
+    if pinned:
+        St, Rt = torch.from_numpy(S).pin_memory(), torch.from_numpy(R).pin_memory()
+        S, R = St.numpy(), Rt.numpy()
+    nwb.nw_fill_batch_host(S, R, 10, 0, 0)
+    for k in range(B):
+        np.testing.assert_array_equal(S[k], want[k])
+
+
 @pytest.mark.parametrize("B,n,tile", [(1, 64, 0), (5, 100, 16), (7, 257, 0), (33, 64, 64), (3, 2048, 0), (4, 700, 128)])
 def test_batch(B, n, tile):
     probs = [inputs.make_problem(n, 10, seed=inputs.pair_seed(k)) for k in range(B)]
