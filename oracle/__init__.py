@@ -57,6 +57,9 @@ def lib() -> ctypes.CDLL:
             L.nw_ref_stream_last.restype = _i32p
             L.nw_ref_stream_free.argtypes = [ctypes.c_void_p]
             L.nw_ref_stream_free.restype = None
+            L.nw_traceback_ref.argtypes = [_i32p, ctypes.c_int64, _i32p, ctypes.c_int64, ctypes.c_int64,
+                                           ctypes.c_int32, ctypes.POINTER(ctypes.c_uint8)]
+            L.nw_traceback_ref.restype = ctypes.c_int64
             _lib = L
     return _lib
 
@@ -79,6 +82,20 @@ def nw_ref(score: np.ndarray, ref: np.ndarray, p: int) -> np.ndarray:
     if rc != 0:
         raise OverflowError("nw_ref: a cell value does not fit in int32")
     return score
+
+
+def nw_traceback_ref(score: np.ndarray, ref: np.ndarray, p: int) -> np.ndarray:
+    """Traceback of a filled ``score`` (NEXT-3): uint8 ops in forward order (0 diagonal, 1 up,
+    2 left; ties diagonal > up > left).  Raises ValueError if a cell matches none of its moves."""
+    assert score.dtype == np.int32 and ref.dtype == np.int32
+    assert score.strides[1] == 4 and ref.strides[1] == 4
+    n = score.shape[0] - 1
+    ops = np.zeros(max(2 * n, 1), dtype=np.uint8)
+    L = lib().nw_traceback_ref(_ptr(score), score.strides[0] // 4, _ptr(ref), ref.strides[0] // 4, n, int(p),
+                               ops.ctypes.data_as(ctypes.POINTER(ctypes.c_uint8)))
+    if L < 0:
+        raise ValueError("nw_traceback_ref: a cell matches none of its three moves")
+    return ops[:L].copy()
 
 
 class NwRefStream:

@@ -98,3 +98,39 @@ void nw_ref_stream_free(void* h) {
   free(s->cur);
   free(s);
 }
+
+/* Traceback (not in the paper — Rodinia's NW stops at the matrix, the
+ * alignment is recovered by walking it back).  Plain definition: from (n,n), at an interior
+ * cell take the first move, in the order diagonal > up > left (reading R12 = SURVEY
+ * C12), whose predecessor reproduces the cell value under the Fig. 2 cell function:
+ *     diagonal  S[i][j] == S[i-1][j-1] + ref[i][j]   op 0 (a_i aligned to b_j)
+ *     up        S[i][j] == S[i-1][j]   - p           op 1 (a_i against a gap)
+ *     left      S[i][j] == S[i][j-1]   - p           op 2 (gap against b_j)
+ * On row 0 / column 0 the path follows the border to the origin (global alignment, C5):
+ * ups while i > 0, lefts while j > 0.  ops[0..L) is written in forward order (origin first).
+ * Returns L, or -1 if some interior cell matches none of its three moves (not a filled
+ * matrix).  int64 arithmetic. */
+int64_t nw_traceback_ref(const int32_t* score, int64_t lds, const int32_t* ref, int64_t ldr, int64_t n,
+                         int32_t p, uint8_t* ops) {
+  uint8_t* back = (uint8_t*)malloc((size_t)(2 * n + 1));
+  if (!back) return -1;
+  int64_t i = n, j = n, L = 0;
+  while (i > 0 && j > 0) {
+    int64_t v = score[i * lds + j];
+    if (v == (int64_t)score[(i - 1) * lds + (j - 1)] + ref[i * ldr + j]) {
+      back[L++] = 0; --i; --j;
+    } else if (v == (int64_t)score[(i - 1) * lds + j] - p) {
+      back[L++] = 1; --i;
+    } else if (v == (int64_t)score[i * lds + (j - 1)] - p) {
+      back[L++] = 2; --j;
+    } else {
+      free(back);
+      return -1;
+    }
+  }
+  while (i > 0) { back[L++] = 1; --i; }
+  while (j > 0) { back[L++] = 2; --j; }
+  for (int64_t k = 0; k < L; ++k) ops[k] = back[L - 1 - k];
+  free(back);
+  return L;
+}

@@ -44,6 +44,12 @@ int nw_ref_stream_rows(void* h, const int32_t* ref_rows, int64_t ldr, const int3
 const int32_t* nw_ref_stream_last(void* h);
 void nw_ref_stream_free(void* h);
 
+/* Traceback of a filled matrix (NEXT-3): ops[0..L) in forward order, 0 = diagonal, 1 = up
+ * (a_i vs gap), 2 = left (gap vs b_j); tie order diagonal > up > left; border cells follow the
+ * border to the origin.  ops needs 2n bytes.  Returns L or -1 (a cell matches no move). */
+int64_t nw_traceback_ref(const int32_t* score, int64_t lds, const int32_t* ref, int64_t ldr, int64_t n,
+                         int32_t p, uint8_t* ops);
+
 #ifdef __cplusplus
 }
 #endif
