@@ -315,6 +315,20 @@ def main():
            "gpu_launches": args.steps * nwb.nw_launch_count({"strip": 0, "seq": 0, "diagonal": 1, "unopt": 2}[args.variant], n, tile),
            "variant": args.variant,
            "clocks": clk.summary()}
+    # ---- NEXT-3: traceback of the filled matrix (outside the timed fill; reported beside it)
+    if not strips and args.variant in ("strip", "seq") and R is not None:
+        SB, RB = (S, R) if B > 1 else (S.unsqueeze(0), R.unsqueeze(0))
+        tb_ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(4)]
+        for e0, e1 in tb_ev:
+            e0.record(stream)
+            ops, length = nwb.nw_traceback_batch(SB, RB, p)
+            e1.record(stream)
+        torch.cuda.synchronize()
+        tb_ms = statistics.median([e0.elapsed_time(e1) for e0, e1 in tb_ev[1:]])
+        steps_total = int(length.to(torch.int64).sum().item())
+        out["traceback"] = {"ms": tb_ms, "pairs": int(SB.shape[0]), "path_steps": steps_total,
+                            "msteps_per_s": steps_total / (tb_ms * 1e-3) / 1e6, "launches": 2,
+                            "bound": "latency (one dependent walk per pair, 33x33 windows)"}
     if args.trace and not strips:
         ntask = (B if B > 1 else 1) * -(-n // nwb.nw_band_width(tile))
         tbuf = torch.zeros(16 * ntask, dtype=torch.int64, device=dev)

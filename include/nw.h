@@ -155,6 +155,27 @@ nw_status nw_fill_host(int32_t* score_host, const int32_t* ref_host, int64_t n, 
 nw_status nw_fill_batch_host(int32_t* score_host, const int32_t* ref_host, int64_t batch, int64_t n,
                              int32_t penalty, int32_t tile, int32_t device);
 
+/* ---- NEXT-3: traceback (the step after the path; not in the paper) -------------------
+ * Recovers the alignment a filled matrix scores.  From (n, n), each interior cell takes the
+ * first move, in the order diagonal > up > left (reading R12), whose predecessor
+ * reproduces its value under the cell function of Fig. 2 / BASELINE north_star:
+ *   op 0 diagonal  S[i][j] == S[i-1][j-1] + ref[i][j]   (a_i aligned to b_j)
+ *   op 1 up        S[i][j] == S[i-1][j] - p             (a_i against a gap)
+ *   op 2 left      S[i][j] == S[i][j-1] - p             (gap against b_j)
+ * On row 0 / column 0 the path follows the border to the origin (global alignment).
+ * score, ref: DEVICE, read-only, the layout of nw_fill_ld (pair k at + k*stride elements).
+ * ops:  DEVICE uint8, >= 2n bytes per pair (pair k at ops + k*ops_stride); on completion
+ *       ops[0..len) holds the path in FORWARD order (origin first); bytes past len undefined.
+ * len:  DEVICE int32 per pair: the path length (n..2n), or -1 if some cell on the walk
+ *       matches none of its three moves (the matrix is not a fill for this ref / p).
+ * ops/len must not overlap each other or score/ref.  Two launches (walk, reverse), enqueued
+ * on `stream`; validation errors are returned synchronously (NW_EINVAL / NW_ERANGE). */
+nw_status nw_traceback(const int32_t* score, int64_t ld_score, const int32_t* ref, int64_t ld_ref, int64_t n,
+                       int32_t penalty, uint8_t* ops, int32_t* len, void* stream);
+nw_status nw_traceback_batch(const int32_t* score, int64_t ld_score, int64_t stride_score, const int32_t* ref,
+                             int64_t ld_ref, int64_t stride_ref, int64_t batch, int64_t n, int32_t penalty,
+                             uint8_t* ops, int64_t ops_stride, int32_t* len, void* stream);
+
 /* ---- the paper's / Rodinia's structure, kept as baselines ----------------------------
  * nw_fill_diagonal: one kernel launch per tile anti-diagonal d = 0..2q-2 (q = ceil(n/b)),
  *   one CTA per b x b tile, the tile staged in shared memory from its LMAD slices Rvert /

@@ -22,7 +22,7 @@ from ._build import LIB_PATH, build  # noqa: F401  (build() is re-exported for _
 
 __all__ = [
     "NwError", "lib", "nw_fill", "nw_fill_batch", "nw_fill_seq", "nw_fill_seq_batch", "nw_fill_sharded", "nw_fill_host", "nw_fill_batch_host",
-    "nw_fill_diagonal", "nw_fill_unopt", "nw_band_width", "nw_launch_count", "nw_diag_lmad",
+    "nw_fill_diagonal", "nw_fill_unopt", "nw_traceback", "nw_traceback_batch", "nw_band_width", "nw_launch_count", "nw_diag_lmad",
     "nw_kernel_info", "nw_strip_map", "nw_debug_set_grid", "nw_debug_set_trace", "nw_release_workspace", "nw_status_str",
 ]
 
@@ -79,6 +79,8 @@ def lib() -> ctypes.CDLL:
             L.nw_fill_batch_host.argtypes = [vp, vp, _i64, _i64, _i32, _i32, _i32]
             L.nw_fill_diagonal.argtypes = [vp, _i64, vp, _i64, _i64, _i32, _i32, vp]
             L.nw_fill_unopt.argtypes = [vp, _i64, vp, _i64, _i64, _i32, _i32, vp]
+            L.nw_traceback.argtypes = [vp, _i64, vp, _i64, _i64, _i32, vp, vp, vp]
+            L.nw_traceback_batch.argtypes = [vp, _i64, _i64, vp, _i64, _i64, _i64, _i64, _i32, vp, _i64, vp, vp]
             L.nw_band_width.argtypes = [_i32]
             L.nw_band_width.restype = _i32
             L.nw_launch_count.argtypes = [_i32, _i64, _i32]
@@ -96,7 +98,7 @@ def lib() -> ctypes.CDLL:
             L.nw_release_workspace.restype = None
             for f in ("nw_fill", "nw_fill_ld", "nw_fill_batch", "nw_fill_batch_ld", "nw_fill_sharded",
                       "nw_fill_host", "nw_fill_batch_host", "nw_fill_diagonal", "nw_fill_unopt", "nw_kernel_info", "nw_fill_seq",
-                      "nw_fill_seq_batch"):
+                      "nw_fill_seq_batch", "nw_traceback", "nw_traceback_batch"):
                 getattr(L, f).restype = ctypes.c_int
             _lib = L
     return _lib
@@ -282,6 +284,34 @@ def nw_fill_diagonal(score, ref, penalty: int, tile: int = 16, stream=None):
 def nw_fill_unopt(score, ref, penalty: int, tile: int = 16, stream=None):
     """The paper's Unopt variant: per diagonal, tiles -> temporary X, then a copy A[W] = X."""
     return _diag("nw_fill_unopt", "nw_fill_unopt", score, ref, penalty, tile, stream)
+
+
+def nw_traceback(score, ref, penalty: int, stream=None):
+    """Traceback of one filled pair (NEXT-3): returns (ops, length) CUDA tensors.
+
+    ops: uint8 (2n,), ops[:length] = the path in forward order (0 diagonal, 1 up, 2 left; ties
+    diagonal > up > left); length: int32 (1,), -1 if the matrix is not a fill of (ref, penalty)."""
+    ops, length = nw_traceback_batch(score.unsqueeze(0), ref.unsqueeze(0), penalty, stream)
+    return ops[0], length
+
+
+def nw_traceback_batch(score, ref, penalty: int, stream=None):
+    """Traceback of B filled pairs: score/ref (B, n+1, >= n+1) -> ops uint8 (B, 2n), length int32 (B,)."""
+    import torch
+    _mat(score, "score"), _mat(ref, "ref")
+    if score.dim() != 3 or ref.dim() != 3 or score.shape[0] != ref.shape[0]:
+        raise ValueError("score/ref must be (B, n+1, >= n+1)")
+    b, n = score.shape[0], score.shape[1] - 1
+    if score.shape[2] < n + 1 or ref.shape[1] < n + 1 or ref.shape[2] < n + 1:
+        raise ValueError("bad batch shapes")
+    ops = torch.empty((b, max(2 * n, 1)), dtype=torch.uint8, device=score.device)
+    length = torch.empty((b,), dtype=torch.int32, device=score.device)
+    with torch.cuda.device(score.device):
+        _check(lib().nw_traceback_batch(score.data_ptr(), score.stride(1), score.stride(0), ref.data_ptr(),
+                                        ref.stride(1), ref.stride(0), b, n, int(penalty), ops.data_ptr(),
+                                        ops.stride(0), length.data_ptr(), _stream_ptr(stream, score.device)),
+               "nw_traceback")
+    return ops, length
 
 
 def nw_band_width(tile: int = 0) -> int:

@@ -15,7 +15,7 @@ CSRC = os.path.join(PKG, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
 LIB_PATH = os.path.join(PKG, "libnwb200.so")
 SOURCES = ["nw_lib.cu"]
-DEPS = ["nw_lib.cu", "nw_common.cuh", "nw_wave.cuh", "nw_diag.cuh", "nw_ptx.cuh"]
+DEPS = ["nw_lib.cu", "nw_common.cuh", "nw_wave.cuh", "nw_diag.cuh", "nw_ptx.cuh", "nw_traceback.cuh"]
 
 NVCC_FLAGS = [
     "-O3", "-std=c++20", "-lineinfo",

@@ -15,6 +15,7 @@
 
 #include "nw.h"
 #include "nw_diag.cuh"
+#include "nw_traceback.cuh"
 #include "nw_wave.cuh"
 
 using namespace nwb200;
@@ -572,6 +573,35 @@ nw_status nw_fill_batch_host(int32_t* score_host, const int32_t* ref_host, int64
 nw_status nw_fill_host(int32_t* score_host, const int32_t* ref_host, int64_t n, int32_t penalty, int32_t tile,
                        int32_t device) {
   return nw_fill_batch_host(score_host, ref_host, 1, n, penalty, tile, device);
+}
+
+nw_status nw_traceback_batch(const int32_t* score, int64_t ld_score, int64_t stride_score, const int32_t* ref,
+                             int64_t ld_ref, int64_t stride_ref, int64_t batch, int64_t n, int32_t penalty,
+                             uint8_t* ops, int64_t ops_stride, int32_t* len, void* stream) {
+  if (batch < 0 || !score || !ref || !ops || !len || n < 0 || n > kMaxN) return NW_EINVAL;
+  if (ld_score < n + 1 || ld_ref < n + 1 || !aligned4(score) || !aligned4(ref) || !aligned4(len)) return NW_EINVAL;
+  if (batch > 1 && (stride_score < span_bytes(n, ld_score) / 4 || stride_ref < span_bytes(n, ld_ref) / 4 ||
+                    ops_stride < 2 * n))
+    return NW_EINVAL;
+  if (batch > 0 && overlaps(ops, (batch - 1) * ops_stride + 2 * n, len, 4 * batch)) return NW_EINVAL;
+  nw_status s = check_range(n, penalty);
+  if (s != NW_OK || batch == 0) return s;
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  TbParams P{score, ld_score, stride_score, ref, ld_ref, stride_ref, batch, n, penalty, ops, ops_stride, len};
+  nw_traceback_kernel<<<static_cast<unsigned>((batch + kTbWarps - 1) / kTbWarps), 32 * kTbWarps, 0, st>>>(P);
+  NW_CU(cudaGetLastError());
+  if (n > 0) {
+    const long long gx = std::min<long long>((n + 255) / 256, 1024);
+    const unsigned gy = static_cast<unsigned>(std::min<long long>(batch, 65535));
+    nw_traceback_reverse_kernel<<<dim3(static_cast<unsigned>(gx), gy), 256, 0, st>>>(ops, ops_stride, len, batch);
+    NW_CU(cudaGetLastError());
+  }
+  return NW_OK;
+}
+
+nw_status nw_traceback(const int32_t* score, int64_t ld_score, const int32_t* ref, int64_t ld_ref, int64_t n,
+                       int32_t penalty, uint8_t* ops, int32_t* len, void* stream) {
+  return nw_traceback_batch(score, ld_score, 0, ref, ld_ref, 0, 1, n, penalty, ops, 2 * n, len, stream);
 }
 
 nw_status nw_fill_diagonal(int32_t* score, int64_t ld_score, const int32_t* ref, int64_t ld_ref, int64_t n,

@@ -139,3 +139,23 @@ def test_sharded_halo_strip_must_end_on_band(L):
 def _has_gpu():
     import torch
     return torch.cuda.is_available()
+
+
+def test_traceback_validation(L):
+    n = 64
+    FAKE_O, FAKE_L = 0x40000000, 0x50000000
+    tb = L.nw_traceback
+    assert tb(None, n + 1, FAKE_R, n + 1, n, 10, FAKE_O, FAKE_L, None) == NW_EINVAL      # null score
+    assert tb(FAKE_S, n + 1, FAKE_R, n + 1, n, 10, None, FAKE_L, None) == NW_EINVAL      # null ops
+    assert tb(FAKE_S, n + 1, FAKE_R, n + 1, n, 10, FAKE_O, None, None) == NW_EINVAL      # null len
+    assert tb(FAKE_S, n, FAKE_R, n + 1, n, 10, FAKE_O, FAKE_L, None) == NW_EINVAL        # ld < n+1
+    assert tb(FAKE_S, n + 1, FAKE_R, n + 1, n, 10, FAKE_O, FAKE_L + 2, None) == NW_EINVAL  # misaligned len
+    assert tb(FAKE_S, n + 1, FAKE_R, n + 1, n, 10, FAKE_O, FAKE_O + 8, None) == NW_EINVAL  # len inside ops
+    assert tb(FAKE_S, n + 1, FAKE_R, n + 1, n, -1, FAKE_O, FAKE_L, None) == NW_ERANGE     # p < 0
+    st = (n + 1) * (n + 1)
+    tbb = L.nw_traceback_batch
+    assert tbb(FAKE_S, n + 1, st, FAKE_R, n + 1, st, 2, n, 10, FAKE_O, 2 * n - 1, FAKE_L, None) == NW_EINVAL
+    assert tbb(FAKE_S, n + 1, st, FAKE_R, n + 1, st, 0, n, 10, FAKE_O, 2 * n, FAKE_L, None) == NW_OK
+    import torch
+    if not torch.cuda.is_available():      # valid arguments, no GPU: fail, never compute on the host
+        assert tb(FAKE_S, n + 1, FAKE_R, n + 1, n, 10, FAKE_O, FAKE_L, None) == NW_ECUDA
