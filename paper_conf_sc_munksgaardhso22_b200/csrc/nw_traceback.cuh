@@ -11,12 +11,15 @@
 // The walk is one dependent chain of up to 2n steps, so a pair is one warp and the design is
 // about latency, not bandwidth (the matrix is read once along a ~33-cell-wide strip around the
 // path: ~2n * 33 * 8 B, negligible next to the fill's 8n^2 B):
-//   * window: the 33 x 33 block of S (and ref) whose bottom-right corner is the current cell is
-//     loaded by the warp in one round of independent coalesced loads;
-//   * the warp then classifies all 32 x 32 interior cells of the window in parallel (one move
-//     code per cell, 3 = no move matches) into shared memory;
+//   * window: the 33-row x 32-column block of S (and ref) whose bottom-right corner is the
+//     current cell; lane c loads column c, all 66 loads of a lane issued before the first use
+//     (one memory round trip per window);
+//   * the warp classifies the window's 32 x 31 interior cells in registers (left / diagonal
+//     neighbours by __shfl_up; int32 differences with an overflow test, exact like the oracle's
+//     int64) into one move code per cell (3 = no move matches) in shared memory;
 //   * lane 0 walks the codes (one LDS per step) until the path leaves the window, which takes
-//     at least 32 steps; the ops go to global memory in traceback order;
+//     at least 31 steps, collecting the ops in shared memory; the warp then stores them to
+//     global memory in traceback order;
 //   * the border tail (all ups or all lefts) is written by the whole warp.
 // A second kernel reverses each pair's ops in place into forward order (one thread per swapped
 // byte pair, grid over the worst case n), so the result matches the oracle's layout.
@@ -25,9 +28,9 @@
 
 namespace nwb200 {
 
-constexpr int kTbWarps = 4;        // pairs per CTA
-constexpr int kTbWin = 32;         // window: (kTbWin+1)^2 cells incl. the predecessor row/column
-constexpr int kTbLd = kTbWin + 1;  // odd pitch: column-wise LDS are bank-conflict free
+constexpr int kTbWarps = 4;   // pairs per CTA
+constexpr int kTbRows = 33;   // window rows i-32 .. i (row 0 of the window = predecessor row)
+constexpr int kTbLd = 33;     // move-code pitch (bytes)
 
 struct TbParams {
   const int32_t* score;
@@ -41,69 +44,78 @@ struct TbParams {
   int32_t* len;          // per pair: path length, or -1 (a cell matches no move)
 };
 
+// x - y == want, exactly (as integers): the int32 difference plus its signed-overflow test
+__device__ __forceinline__ bool diff_is(int32_t x, int32_t y, int32_t want) {
+  const int32_t d = static_cast<int32_t>(static_cast<uint32_t>(x) - static_cast<uint32_t>(y));
+  return d == want && ((x ^ y) & (x ^ d)) >= 0;
+}
+
 __global__ void __launch_bounds__(32 * kTbWarps) nw_traceback_kernel(TbParams P) {
-  __shared__ int32_t sS[kTbWarps][kTbLd * kTbLd];
-  __shared__ int32_t sR[kTbWarps][kTbLd * kTbLd];
-  __shared__ uint8_t sM[kTbWarps][kTbLd * kTbLd];
+  __shared__ uint8_t sM[kTbWarps][kTbRows * kTbLd];
+  __shared__ uint8_t sO[kTbWarps][2 * kTbRows];
   const int wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const long long pair = static_cast<long long>(blockIdx.x) * kTbWarps + wid;
   if (pair >= P.batch) return;
   const int32_t* __restrict__ S = P.score + pair * P.pss;
   const int32_t* __restrict__ R = P.ref + pair * P.psr;
   uint8_t* __restrict__ ops = P.ops + pair * P.ops_stride;
-  int32_t* ws = sS[wid];
-  int32_t* wr = sR[wid];
   uint8_t* wm = sM[wid];
-  const long long p = P.p;
+  uint8_t* wo = sO[wid];
+  const int32_t p = P.p;
 
   long long i = P.n, j = P.n, L = 0;
   int bad = 0;
   while (i > 0 && j > 0) {
-    const long long i0 = i > kTbWin ? i - kTbWin : 0, j0 = j > kTbWin ? j - kTbWin : 0;
+    // window: rows i0..i (<= 33), columns j0..j (<= 32, lane c holds column j0 + c).  Rows and
+    // columns past the window are clamped to it (valid addresses; their codes are never read).
+    const long long i0 = i > kTbRows - 1 ? i - (kTbRows - 1) : 0, j0 = j > 31 ? j - 31 : 0;
     const int h = static_cast<int>(i - i0) + 1, w = static_cast<int>(j - j0) + 1;
-    // one round of independent loads: row r of the window, lanes across the columns
-    for (int e = lane; e < h * kTbLd; e += 32) {
-      const int r = e / kTbLd, c = e - r * kTbLd;
-      if (c < w) {
-        ws[r * kTbLd + c] = __ldg(S + (i0 + r) * P.lds + j0 + c);
-        wr[r * kTbLd + c] = __ldg(R + (i0 + r) * P.ldr + j0 + c);
-      }
+    const int c = lane < w ? lane : w - 1;
+    const int32_t* sp = S + i0 * P.lds + j0 + c;
+    const int32_t* rp = R + i0 * P.ldr + j0 + c;
+    // one round of independent loads (all issued before the first use)
+    int32_t vs[kTbRows], vr[kTbRows];
+#pragma unroll
+    for (int r = 0; r < kTbRows; ++r) {
+      const int rr = r < h ? r : h - 1;
+      vs[r] = __ldg(sp + rr * P.lds);
+      if (r >= 1) vr[r] = __ldg(rp + rr * P.ldr);
+    }
+    // move code of every cell (row r >= 1, column lane >= 1): left / diagonal neighbours from
+    // lane - 1 by shuffle
+    int32_t diag = __shfl_up_sync(0xffffffffu, vs[0], 1);
+#pragma unroll
+    for (int r = 1; r < kTbRows; ++r) {
+      const int32_t left = __shfl_up_sync(0xffffffffu, vs[r], 1);
+      const int32_t v = vs[r];
+      const uint8_t m = diff_is(v, diag, vr[r]) ? 0 : diff_is(vs[r - 1], v, p) ? 1 : diff_is(left, v, p) ? 2 : 3;
+      wm[r * kTbLd + lane] = m;
+      diag = left;
     }
     __syncwarp();
-    // classify every interior cell of the window (rows/cols >= 1 of the window)
-    for (int e = lane; e < (h - 1) * kTbLd; e += 32) {
-      const int r = 1 + e / kTbLd, c = e - (r - 1) * kTbLd;
-      if (c >= 1 && c < w) {
-        const long long v = ws[r * kTbLd + c];
-        uint8_t m = 3;
-        if (v == static_cast<long long>(ws[(r - 1) * kTbLd + c - 1]) + wr[r * kTbLd + c]) m = 0;
-        else if (v == static_cast<long long>(ws[(r - 1) * kTbLd + c]) - p) m = 1;
-        else if (v == static_cast<long long>(ws[r * kTbLd + c - 1]) - p) m = 2;
-        wm[r * kTbLd + c] = m;
-      }
-    }
-    __syncwarp();
+    int k = 0;
     if (lane == 0) {
       int ci = h - 1, cj = w - 1;
-      long long l = L;
       while (ci > 0 && cj > 0) {
         const uint8_t m = wm[ci * kTbLd + cj];
         if (m == 3) {
           bad = 1;
           break;
         }
-        ops[l++] = m;
+        wo[k++] = m;
         ci -= (m != 2);
         cj -= (m != 1);
       }
       i = i0 + ci;
       j = j0 + cj;
-      L = l;
     }
     i = __shfl_sync(0xffffffffu, i, 0);
     j = __shfl_sync(0xffffffffu, j, 0);
-    L = __shfl_sync(0xffffffffu, L, 0);
+    k = __shfl_sync(0xffffffffu, k, 0);
     bad = __shfl_sync(0xffffffffu, bad, 0);
+    __syncwarp();
+    for (int e = lane; e < k; e += 32) ops[L + e] = wo[e];
+    L += k;
     __syncwarp();
     if (bad) break;
   }
@@ -112,7 +124,7 @@ __global__ void __launch_bounds__(32 * kTbWarps) nw_traceback_kernel(TbParams P)
     return;
   }
   // border tail, traceback order: i ups (column 0), then j lefts (row 0); one of them is 0
-  for (long long k = lane; k < i + j; k += 32) ops[L + k] = k < i ? 1 : 2;
+  for (long long e = lane; e < i + j; e += 32) ops[L + e] = e < i ? 1 : 2;
   if (lane == 0) P.len[pair] = static_cast<int32_t>(L + i + j);
 }
 
