@@ -17,7 +17,8 @@
 //   * the warp classifies the window's 32 x 31 interior cells in registers (left / diagonal
 //     neighbours by __shfl_up; int32 differences with an overflow test, exact like the oracle's
 //     int64) into one move code per cell (3 = no move matches) in shared memory;
-//   * lane 0 walks the codes (one LDS per step) until the path leaves the window, which takes
+//   * lane 0 walks the codes (each code is the move's address step, so a step is one
+//     LDS -> IADD chain; row/column 0 of the window hold a stop code) until the path leaves the window, which takes
 //     at least 31 steps, collecting the ops in shared memory; the warp then stores them to
 //     global memory in traceback order;
 //   * the border tail (all ups or all lefts) is written by the whole warp.
@@ -28,9 +29,14 @@
 
 namespace nwb200 {
 
-constexpr int kTbWarps = 4;   // pairs per CTA
+constexpr int kTbWarps = 4;   // warps per CTA
+constexpr int kTbFewPairs = 296;  // up to 2 x 148 pairs: one pair per CTA (4 warps per pair)
 constexpr int kTbRows = 33;   // window rows i-32 .. i (row 0 of the window = predecessor row)
 constexpr int kTbLd = 33;     // move-code pitch (bytes)
+// move codes in shared memory = the address step of the move in the code array
+constexpr uint8_t kTbDiag = kTbLd + 1, kTbUp = kTbLd, kTbLeft = 1;
+constexpr uint8_t kTbBad = 0xFE;   // no move reproduces the cell
+constexpr uint8_t kTbStop = 0xFF;  // window row 0 / column 0: the path leaves the window
 
 struct TbParams {
   const int32_t* score;
@@ -50,19 +56,33 @@ __device__ __forceinline__ bool diff_is(int32_t x, int32_t y, int32_t want) {
   return d == want && ((x ^ y) & (x ^ d)) >= 0;
 }
 
+// WPP warps per pair (1 for large batches: kTbWarps pairs per CTA; 4 for few pairs: the
+// window's rows are loaded and classified by four warps, 8 rows each, and lane 0 of the first
+// warp walks).  The group synchronises with a named barrier (id = group + 1).
+template <int WPP>
 __global__ void __launch_bounds__(32 * kTbWarps) nw_traceback_kernel(TbParams P) {
-  __shared__ uint8_t sM[kTbWarps][kTbRows * kTbLd];
-  __shared__ uint8_t sO[kTbWarps][2 * kTbRows];
+  constexpr int G = kTbWarps / WPP;          // pairs per CTA
+  constexpr int RPW = (kTbRows - 1) / WPP;   // window rows classified per warp
+  __shared__ uint8_t sM[G][kTbRows * kTbLd];
+  __shared__ uint8_t sO[G][2 * kTbRows];
+  __shared__ long long sIJ[G][2];
+  __shared__ int sK[G], sBad[G];
   const int wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const long long pair = static_cast<long long>(blockIdx.x) * kTbWarps + wid;
-  if (pair >= P.batch) return;
+  const int g = wid / WPP, sub = wid - g * WPP;
+  const long long pair = static_cast<long long>(blockIdx.x) * G + g;
+  if (pair >= P.batch) return;  // the whole group (same pair) leaves together
   const int32_t* __restrict__ S = P.score + pair * P.pss;
   const int32_t* __restrict__ R = P.ref + pair * P.psr;
   uint8_t* __restrict__ ops = P.ops + pair * P.ops_stride;
-  uint8_t* wm = sM[wid];
-  uint8_t* wo = sO[wid];
+  uint8_t* wm = sM[g];
+  uint8_t* wo = sO[g];
   const int32_t p = P.p;
+  auto group_sync = [&]() {
+    if constexpr (WPP == 1) __syncwarp();
+    else asm volatile("bar.sync %0, %1;" ::"r"(g + 1), "r"(32 * WPP) : "memory");
+  };
 
+  if (sub == 0) wm[lane] = kTbStop;  // window row 0 (the predecessor row) stops the walk; column 0 below
   long long i = P.n, j = P.n, L = 0;
   int bad = 0;
   while (i > 0 && j > 0) {
@@ -71,54 +91,55 @@ __global__ void __launch_bounds__(32 * kTbWarps) nw_traceback_kernel(TbParams P)
     const long long i0 = i > kTbRows - 1 ? i - (kTbRows - 1) : 0, j0 = j > 31 ? j - 31 : 0;
     const int h = static_cast<int>(i - i0) + 1, w = static_cast<int>(j - j0) + 1;
     const int c = lane < w ? lane : w - 1;
+    const int rb = sub * RPW;  // this warp loads window rows rb .. rb + RPW, classifies rb+1 ..
     const int32_t* sp = S + i0 * P.lds + j0 + c;
     const int32_t* rp = R + i0 * P.ldr + j0 + c;
     // one round of independent loads (all issued before the first use)
-    int32_t vs[kTbRows], vr[kTbRows];
+    int32_t vs[RPW + 1], vr[RPW + 1];
 #pragma unroll
-    for (int r = 0; r < kTbRows; ++r) {
-      const int rr = r < h ? r : h - 1;
-      vs[r] = __ldg(sp + rr * P.lds);
-      if (r >= 1) vr[r] = __ldg(rp + rr * P.ldr);
+    for (int q = 0; q <= RPW; ++q) {
+      const int rr = rb + q < h ? rb + q : h - 1;
+      vs[q] = __ldg(sp + rr * P.lds);
+      if (q >= 1) vr[q] = __ldg(rp + rr * P.ldr);
     }
-    // move code of every cell (row r >= 1, column lane >= 1): left / diagonal neighbours from
+    // move code of every cell (row >= 1, column lane >= 1): left / diagonal neighbours from
     // lane - 1 by shuffle
     int32_t diag = __shfl_up_sync(0xffffffffu, vs[0], 1);
 #pragma unroll
-    for (int r = 1; r < kTbRows; ++r) {
-      const int32_t left = __shfl_up_sync(0xffffffffu, vs[r], 1);
-      const int32_t v = vs[r];
-      const uint8_t m = diff_is(v, diag, vr[r]) ? 0 : diff_is(vs[r - 1], v, p) ? 1 : diff_is(left, v, p) ? 2 : 3;
-      wm[r * kTbLd + lane] = m;
+    for (int q = 1; q <= RPW; ++q) {
+      const int32_t left = __shfl_up_sync(0xffffffffu, vs[q], 1);
+      const int32_t v = vs[q];
+      const uint8_t m = diff_is(v, diag, vr[q]) ? kTbDiag : diff_is(vs[q - 1], v, p) ? kTbUp
+                      : diff_is(left, v, p) ? kTbLeft : kTbBad;
+      wm[(rb + q) * kTbLd + lane] = lane == 0 ? kTbStop : m;
       diag = left;
     }
-    __syncwarp();
-    int k = 0;
-    if (lane == 0) {
-      int ci = h - 1, cj = w - 1;
-      while (ci > 0 && cj > 0) {
-        const uint8_t m = wm[ci * kTbLd + cj];
-        if (m == 3) {
-          bad = 1;
-          break;
-        }
+    group_sync();
+    if (sub == 0 && lane == 0) {
+      // the code is the address step: one LDS -> IADD -> LDS chain per step
+      int a = (h - 1) * kTbLd + (w - 1), k = 0;
+      uint8_t m;
+      while ((m = wm[a]) < kTbBad) {
         wo[k++] = m;
-        ci -= (m != 2);
-        cj -= (m != 1);
+        a -= m;
       }
-      i = i0 + ci;
-      j = j0 + cj;
+      const int ci = a / kTbLd;
+      sIJ[g][0] = i0 + ci;
+      sIJ[g][1] = j0 + (a - ci * kTbLd);
+      sK[g] = k;
+      sBad[g] = m == kTbBad;
     }
-    i = __shfl_sync(0xffffffffu, i, 0);
-    j = __shfl_sync(0xffffffffu, j, 0);
-    k = __shfl_sync(0xffffffffu, k, 0);
-    bad = __shfl_sync(0xffffffffu, bad, 0);
-    __syncwarp();
-    for (int e = lane; e < k; e += 32) ops[L + e] = wo[e];
+    group_sync();
+    i = sIJ[g][0];
+    j = sIJ[g][1];
+    bad = sBad[g];
+    const int k = sK[g];
+    if (sub == 0)
+      for (int e = lane; e < k; e += 32) ops[L + e] = wo[e] == kTbDiag ? 0 : (wo[e] == kTbUp ? 1 : 2);
     L += k;
-    __syncwarp();
     if (bad) break;
   }
+  if (sub != 0) return;
   if (bad) {
     if (lane == 0) P.len[pair] = -1;
     return;

@@ -74,7 +74,7 @@ def test_traceback_corrupted_matrix():
     assert L == -1
 
 
-@pytest.mark.parametrize("B,n", [(7, 64), (33, 129)])
+@pytest.mark.parametrize("B,n", [(7, 64), (33, 129), (300, 40), (1100, 17)])   # > 296: one warp per pair
 def test_traceback_batch_after_device_fill(B, n):
     p = 10
     pairs = [inputs.make_problem(n, p, seed=inputs.pair_seed(k)) for k in range(B)]
