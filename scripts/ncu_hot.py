@@ -5,7 +5,7 @@ top = int(sys.argv[2]) if len(sys.argv) > 2 else 40
 out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass"], capture_output=True, text=True).stdout
 rows = list(csv.reader(io.StringIO(out)))
 h = rows[1]
-data = rows[2:]
+data = [x for x in rows[2:] if len(x) > 1 and (x[h.index("Warp Stall Sampling (All Samples)")] or "0").isdigit()]
 i_s = h.index("Warp Stall Sampling (All Samples)"); i_src = h.index("Source"); i_ex = h.index("Instructions Executed")
 stall_cols = [i for i, x in enumerate(h) if x.startswith("stall_") or "Stall" in x and i != i_s]
 tot = sum(int(x[i_s] or 0) for x in data)
