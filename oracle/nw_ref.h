@@ -16,7 +16,9 @@
  * Pins (tests/test_oracle.py): hand example (tests/golden/appendix_b.txt), brute-force
  * enumeration of all alignments for n <= 8 (standard and arbitrary borders), the
  * constant-ref closed form, border-shift / transpose metamorphics, bounds, and an
- * independent max-plus prefix-scan formulation.  Every function here is pinned.
+ * independent max-plus prefix-scan formulation.  nw_traceback_ref is pinned separately
+ * (tests/test_traceback_oracle.py): hand example, brute force over every alignment for n <= 6
+ * with the tie rule, and the path's independently summed score.  Every function here is pinned.
  */
 #ifndef NW_REF_H
 #define NW_REF_H

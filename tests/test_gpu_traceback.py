@@ -24,6 +24,8 @@ def problem(n, p, seed, family):
         ref[1:, 1:] = rng.integers(-1, 2, size=(n, n))
         score = inputs.init_borders(inputs.aligned_matrix(n), p)
         return score, ref
+    if family == "borders":        # arbitrary row 0 / column 0 (reading R5)
+        return inputs.make_problem(n, p, seed=seed, border_seed=seed + 1)
     return inputs.make_problem(n, p, seed=seed, family=family)
 
 
@@ -36,7 +38,7 @@ def run_gpu(score, ref, p):
 
 @pytest.mark.parametrize("n", [1, 2, 5, 31, 32, 33, 64, 65, 100, 257, 1000, 2048])
 @pytest.mark.parametrize("p,family", [(10, "random"), (3, "homologous"), (0, "ties"), (1, "ties"),
-                                      (1000, "random")])
+                                      (1000, "random"), (10, "borders"), (0, "const")])
 def test_traceback_matches_oracle(n, p, family):
     score, ref = problem(n, p, n + p, family)
     oracle.nw_ref(score, ref, p)
