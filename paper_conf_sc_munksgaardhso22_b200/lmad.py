@@ -149,3 +149,34 @@ def nw_schedule_proofs(lib, n: int, tile: int, ld: int | None = None):
         W, Rv, Rh = nw_diag_lmads(lib, n, ld, tile, d)
         res.append((d, non_overlap(W, Rv), non_overlap(W, Rh)))
     return res
+
+
+def wave_band_lmads(n: int, ld: int, width: int, k: int):
+    """(W, Rleft, Rtop) of band k of the persistent kernel (csrc/nw_wave.cuh): columns
+    c0 = k*width + 1 .. c1 = min((k+1)*width, n), all rows.  The band writes the interior of its
+    columns, reads the column left of it (rows 0..n: the border, or band k-1's last column) and
+    row 0 of its columns."""
+    c0, c1 = k * width + 1, min((k + 1) * width, n)
+    W = Lmad(ld + c0, ((n, ld), (c1 - c0 + 1, 1)))
+    Rleft = Lmad(c0 - 1, ((n + 1, ld),))
+    Rtop = Lmad(c0, ((c1 - c0 + 1, 1),))
+    return W, Rleft, Rtop
+
+
+def wave_schedule_proofs(n: int, width: int, ld: int | None = None):
+    """The persistent kernel runs neighbouring bands concurrently, in place.  Legal iff, for every
+    band k: its writes miss its own reads (W_k ∩ Rleft_k = W_k ∩ Rtop_k = ∅), no two bands write
+    one cell (W_k ∩ W_k+1 = ∅), and band k+1 never overwrites what band k still reads
+    (W_k+1 ∩ Rleft_k = W_k+1 ∩ Rtop_k = ∅).  Returns one tuple of five proofs per band."""
+    ld = n + 1 if ld is None else ld
+    nb = -(-n // width)
+    res = []
+    for k in range(nb):
+        W, Rl, Rt = wave_band_lmads(n, ld, width, k)
+        if k + 1 < nb:
+            W1 = wave_band_lmads(n, ld, width, k + 1)[0]
+            nxt = (non_overlap(W, W1), non_overlap(W1, Rl), non_overlap(W1, Rt))
+        else:
+            nxt = (True, True, True)
+        res.append((non_overlap(W, Rl), non_overlap(W, Rt)) + nxt)
+    return res

@@ -6,6 +6,9 @@ L1  Fig. 9: W ∩ Rvert = ∅ and W ∩ Rhoriz = ∅ are PROVEN fo
     enumeration of the point sets agrees.
 L2  soundness: on random small LMAD pairs, every "proven disjoint" answer is confirmed by
     enumerating both point sets; overlapping pairs are never proven.
+L4  the persistent kernel's bands (wave_band_lmads): every band's writes miss its reads, the
+    next band's writes miss this band's reads and writes (brute force agrees on small n), and
+    the true dependency (band k+1 reads band k's last column) is not proven disjoint.
 L3  the schedule the diagonal kernels run (nw_diag_lmad of the C ABI, host-only): every tile
     anti-diagonal's write set is proven disjoint from its read sets, while the NEXT diagonal's
     Rvert / Rhoriz do overlap W (they read what W wrote) and are not proven.
@@ -15,7 +18,8 @@ import random
 import pytest
 
 import paper_conf_sc_munksgaardhso22_b200 as nwb
-from paper_conf_sc_munksgaardhso22_b200.lmad import Lmad, non_overlap, nw_diag_lmads, nw_schedule_proofs
+from paper_conf_sc_munksgaardhso22_b200.lmad import (Lmad, non_overlap, nw_diag_lmads, nw_schedule_proofs,
+                                                    wave_band_lmads, wave_schedule_proofs)
 
 
 def points(L):
@@ -70,3 +74,23 @@ def test_next_diagonal_reads_are_not_disjoint(n, tile):
         _, Rv1, Rh1 = nw_diag_lmads(L, n, n + 1, tile, d + 1)
         assert points(W) & (points(Rv1) | points(Rh1))          # d+1 consumes d's results
         assert not (non_overlap(W, Rv1) and non_overlap(W, Rh1))
+
+
+@pytest.mark.parametrize("n,width", [(40, 8), (100, 32), (1000, 128), (32768, 256), (33000, 256)])
+def test_wave_bands_proven(n, width):
+    res = wave_schedule_proofs(n, width)
+    assert all(all(r) for r in res), [k for k, r in enumerate(res) if not all(r)]
+    if n <= 100:
+        for k in range(len(res) - 1):
+            W, Rl, Rt = wave_band_lmads(n, n + 1, width, k)
+            W1, Rl1, _ = wave_band_lmads(n, n + 1, width, k + 1)
+            assert not (points(W) & (points(Rl) | points(Rt) | points(W1)))
+            assert not (points(W1) & (points(Rl) | points(Rt)))
+            assert points(W) & points(Rl1)                    # k+1 reads k's last column
+            assert not non_overlap(W, Rl1)
+
+
+def test_wave_bands_use_the_library_width():
+    for tile in (0, 16, 64):
+        w = nwb.nw_band_width(tile)
+        assert all(all(r) for r in wave_schedule_proofs(4096, w))
