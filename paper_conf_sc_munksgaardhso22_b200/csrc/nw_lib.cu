@@ -589,7 +589,7 @@ nw_status nw_traceback_batch(const int32_t* score, int64_t ld_score, int64_t str
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   TbParams P{score, ld_score, stride_score, ref, ld_ref, stride_ref, batch, n, penalty, ops, ops_stride, len};
   if (batch <= kTbFewPairs)  // few pairs: four warps share each window
-    nw_traceback_kernel<4><<<static_cast<unsigned>(batch), 32 * kTbWarps, 0, st>>>(P);
+    nw_traceback_kernel<kTbFewWpp, kTbFewWpp><<<static_cast<unsigned>(batch), 32 * kTbFewWpp, 0, st>>>(P);
   else
     nw_traceback_kernel<1><<<static_cast<unsigned>((batch + kTbWarps - 1) / kTbWarps), 32 * kTbWarps, 0, st>>>(P);
   NW_CU(cudaGetLastError());
