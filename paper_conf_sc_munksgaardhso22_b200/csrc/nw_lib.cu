@@ -588,7 +588,7 @@ nw_status nw_traceback_batch(const int32_t* score, int64_t ld_score, int64_t str
   if (s != NW_OK || batch == 0) return s;
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   TbParams P{score, ld_score, stride_score, ref, ld_ref, stride_ref, batch, n, penalty, ops, ops_stride, len};
-  if (batch <= kTbFewPairs)  // few pairs: four warps share each window
+  if (batch <= kTbFewPairs)  // few pairs: kTbFewWpp warps share each window
     nw_traceback_kernel<kTbFewWpp, kTbFewWpp><<<static_cast<unsigned>(batch), 32 * kTbFewWpp, 0, st>>>(P);
   else
     nw_traceback_kernel<1><<<static_cast<unsigned>((batch + kTbWarps - 1) / kTbWarps), 32 * kTbWarps, 0, st>>>(P);

@@ -32,7 +32,7 @@ namespace nwb200 {
 constexpr int kTbWarps = 4;   // warps per CTA
 constexpr int kTbFewPairs = 296;  // up to 2 x 148 pairs: one pair per CTA
 #ifndef NW_TB_FEW_WPP
-#define NW_TB_FEW_WPP 8
+#define NW_TB_FEW_WPP 16
 #endif
 constexpr int kTbFewWpp = NW_TB_FEW_WPP;  // warps per pair (and per CTA) for few pairs
 constexpr int kTbRows = 33;   // window rows i-32 .. i (row 0 of the window = predecessor row)
@@ -61,7 +61,7 @@ __device__ __forceinline__ bool diff_is(int32_t x, int32_t y, int32_t want) {
 }
 
 // WPP warps per pair (1 for large batches: kTbWarps pairs per CTA; 4 for few pairs: the
-// window's rows are loaded and classified by four warps, 8 rows each, and lane 0 of the first
+// window's rows are loaded and classified by kTbFewWpp = 16 warps, 2 rows each, and lane 0 of the first
 // warp walks).  The group synchronises with a named barrier (id = group + 1).
 template <int WPP, int NW = kTbWarps>
 __global__ void __launch_bounds__(32 * NW) nw_traceback_kernel(TbParams P) {
