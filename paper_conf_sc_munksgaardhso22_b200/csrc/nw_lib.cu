@@ -583,7 +583,14 @@ nw_status nw_traceback_batch(const int32_t* score, int64_t ld_score, int64_t str
   if (batch > 1 && (stride_score < span_bytes(n, ld_score) / 4 || stride_ref < span_bytes(n, ld_ref) / 4 ||
                     ops_stride < 2 * n))
     return NW_EINVAL;
-  if (batch > 0 && overlaps(ops, (batch - 1) * ops_stride + 2 * n, len, 4 * batch)) return NW_EINVAL;
+  if (batch > 0) {  // outputs must not overlap each other or the inputs
+    const int64_t ob = (batch - 1) * ops_stride + 2 * n, lb = 4 * batch;
+    const int64_t sb = 4 * ((batch - 1) * stride_score) + span_bytes(n, ld_score);
+    const int64_t rb = 4 * ((batch - 1) * stride_ref) + span_bytes(n, ld_ref);
+    if (overlaps(ops, ob, len, lb) || overlaps(ops, ob, score, sb) || overlaps(ops, ob, ref, rb) ||
+        overlaps(len, lb, score, sb) || overlaps(len, lb, ref, rb))
+      return NW_EINVAL;
+  }
   nw_status s = check_range(n, penalty);
   if (s != NW_OK || batch == 0) return s;
   cudaStream_t st = static_cast<cudaStream_t>(stream);

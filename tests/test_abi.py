@@ -152,6 +152,8 @@ def test_traceback_validation(L):
     assert tb(FAKE_S, n + 1, FAKE_R, n + 1, n, 10, FAKE_O, FAKE_L + 2, None) == NW_EINVAL  # misaligned len
     assert tb(FAKE_S, n + 1, FAKE_R, n + 1, n, 10, FAKE_O, FAKE_O + 8, None) == NW_EINVAL  # len inside ops
     assert tb(FAKE_S, n + 1, FAKE_R, n + 1, n, -1, FAKE_O, FAKE_L, None) == NW_ERANGE     # p < 0
+    assert tb(FAKE_S, n + 1, FAKE_R, n + 1, n, 10, FAKE_S + 64, FAKE_L, None) == NW_EINVAL  # ops inside score
+    assert tb(FAKE_S, n + 1, FAKE_R, n + 1, n, 10, FAKE_O, FAKE_R + 64, None) == NW_EINVAL  # len inside ref
     st = (n + 1) * (n + 1)
     tbb = L.nw_traceback_batch
     assert tbb(FAKE_S, n + 1, st, FAKE_R, n + 1, st, 2, n, 10, FAKE_O, 2 * n - 1, FAKE_L, None) == NW_EINVAL
