@@ -598,7 +598,8 @@ nw_status nw_traceback_batch(const int32_t* score, int64_t ld_score, int64_t str
   if (batch <= kTbFewPairs)  // few pairs: kTbFewWpp warps share each window
     nw_traceback_kernel<kTbFewWpp, kTbFewWpp><<<static_cast<unsigned>(batch), 32 * kTbFewWpp, 0, st>>>(P);
   else
-    nw_traceback_kernel<1><<<static_cast<unsigned>((batch + kTbWarps - 1) / kTbWarps), 32 * kTbWarps, 0, st>>>(P);
+    nw_traceback_kernel<kTbManyWpp><<<static_cast<unsigned>((batch * kTbManyWpp + kTbWarps - 1) / kTbWarps),
+                                      32 * kTbWarps, 0, st>>>(P);
   NW_CU(cudaGetLastError());
   if (n > 0) {
     const long long gx = std::min<long long>((n + 255) / 256, 1024);

@@ -35,6 +35,10 @@ constexpr int kTbFewPairs = 296;  // up to 2 x 148 pairs: one pair per CTA
 #define NW_TB_FEW_WPP 16
 #endif
 constexpr int kTbFewWpp = NW_TB_FEW_WPP;  // warps per pair (and per CTA) for few pairs
+#ifndef NW_TB_MANY_WPP
+#define NW_TB_MANY_WPP 1
+#endif
+constexpr int kTbManyWpp = NW_TB_MANY_WPP;  // warps per pair for many pairs
 constexpr int kTbRows = 33;   // window rows i-32 .. i (row 0 of the window = predecessor row)
 constexpr int kTbLd = 33;     // move-code pitch (bytes)
 // move codes in shared memory = the address step of the move in the code array
