@@ -187,6 +187,8 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--layout", default="rodinia", choices=["rodinia", "aligned"],
+                    help="matrix layout: pitch n+1 (Rodinia) or 16-byte aligned interior rows")
     ap.add_argument("--trace", default="", help="write per-band {task,start,end,smid} of one extra launch here (.npy)")
     ap.add_argument("--variant", default="strip", choices=["strip", "diagonal", "unopt", "seq"],
                     help="ablation: the paper's per-diagonal structure (Opt) / Unopt instead of the "
@@ -240,7 +242,7 @@ def main():
             nwb.nw_fill_batch(S, R, p, tile)
         cells_local = nb * n * n
     else:
-        S, R = inputs.device_problem(n, p, device=dev)
+        S, R = inputs.device_problem(n, p, device=dev, layout=args.layout)
         if args.variant == "seq":       # NEXT-2: ref generated on chip from the sequences
             a_h, b_h = inputs.gen_pair(n, inputs.SEED)
             Ad, Bd = torch.from_numpy(a_h).to(dev), torch.from_numpy(b_h).to(dev)

@@ -176,8 +176,17 @@ def make_problem(n: int, p: int = 10, seed: int = SEED, family: str = "random", 
     return score, ref
 
 
+def device_aligned_matrix(n: int, device="cuda"):
+    """An (n+1) x (n+1) int32 CUDA view whose interior rows start 16-byte aligned: pitch a multiple of 4
+    elements and element (0, 1) on a 16-byte boundary (a layout, no data)."""
+    import torch
+    ld = (n + 1 + 3) & ~3
+    buf = torch.empty((n + 1) * ld + 4, dtype=torch.int32, device=device)
+    return buf[3:3 + (n + 1) * ld].view(n + 1, ld)[:, : n + 1]
+
+
 def device_problem(n: int, p: int = 10, seed: int = SEED, device="cuda", score=None, ref=None,
-                   sentinel: bool = True, chunk_rows: int = 4096):
+                   sentinel: bool = True, chunk_rows: int = 4096, layout: str = "rodinia"):
     """The same Rodinia-style problem as make_problem(n, p, seed), built ON THE DEVICE (for the
     large bench configs): sequences from the C splitmix64 generator, ref = B62[a_i][b_j] by a
     table gather in row chunks, global-alignment borders.  Optionally fills preallocated
@@ -188,9 +197,9 @@ def device_problem(n: int, p: int = 10, seed: int = SEED, device="cuda", score=N
     ta = torch.from_numpy(a.astype(np.int64)).to(device)
     tb = torch.from_numpy(b.astype(np.int64)).to(device)
     if score is None:
-        score = torch.empty((n + 1, n + 1), dtype=torch.int32, device=device)
+        score = device_aligned_matrix(n, device) if layout == "aligned" else torch.empty((n + 1, n + 1), dtype=torch.int32, device=device)
     if ref is None:
-        ref = torch.empty((n + 1, n + 1), dtype=torch.int32, device=device)
+        ref = device_aligned_matrix(n, device) if layout == "aligned" else torch.empty((n + 1, n + 1), dtype=torch.int32, device=device)
     ref[0, : n + 1] = 0
     ref[:, 0] = 0
     rows_b = table[:, tb]                       # (24, n): B62[x][b_j] for every residue x

@@ -37,10 +37,10 @@ def expect(score, ref, p):
     return oracle.nw_ref(score.copy(), ref, p)
 
 
-def gpu_fill(score, ref, p, tile, fn=None, ld=None, offset=0):
+def gpu_fill(score, ref, p, tile, fn=None, ld=None, offset=0, ref_offset=None):
     n = score.shape[0] - 1
     s = to_dev(score, ld, offset)
-    r = to_dev(ref, ld, (offset * 3) % 4)
+    r = to_dev(ref, ld, (offset * 3) % 4 if ref_offset is None else ref_offset)
     (fn or nwb.nw_fill)(s, r, p, tile)
     torch.cuda.synchronize()
     return s[:, : n + 1].cpu().numpy()
@@ -73,6 +73,16 @@ def test_fill_pitch_and_alignment(ld_extra, offset):
     n = 517
     score, ref = inputs.make_problem(n, 10, seed=11)
     got = gpu_fill(score, ref, 10, 0, ld=n + 1 + ld_extra, offset=offset)
+    np.testing.assert_array_equal(got, expect(score, ref, 10))
+
+
+@pytest.mark.parametrize("tile", [0, 128])
+@pytest.mark.parametrize("n", [1, 2, 17, 100, 128, 129, 257, 1000, 1024, 1531])
+def test_fill_aligned_layout(n, tile):
+    """16-byte aligned interior rows (pitch 0 mod 4, element (0, 1) on a 16-byte boundary)."""
+    score, ref = inputs.make_problem(n, 10, seed=100 + n)
+    ld = (n + 1 + 3) & ~3
+    got = gpu_fill(score, ref, 10, tile, ld=ld, offset=3, ref_offset=3)
     np.testing.assert_array_equal(got, expect(score, ref, 10))
 
 
