@@ -37,8 +37,10 @@
  *     The result does not depend on it (R8).
  *   - Any n >= 0 is accepted (ragged last band: n need not be a multiple of b).
  *   - Validation is synchronous and happens before anything is enqueued.  Range contract:
- *     0 <= penalty and 2*n*penalty + n*NW_REF_MAX < 2^31 (else NW_ERANGE), |ref| <= NW_REF_MAX
- *     and |border| <= 2^30 are the caller's promise (int32 arithmetic cannot overflow then).
+ *     0 <= penalty and (n+1)*(2*penalty + NW_REF_MAX) < 2^30 (else NW_ERANGE); |ref| <= NW_REF_MAX
+ *     and |border| <= 2^30 are the caller's promise.  Then every intermediate of the kernels'
+ *     gap-normalised arithmetic (S + (i+j)*p, bounded by |border| + (n+1)*(2p + NW_REF_MAX))
+ *     fits int32, and so does every cell (reading R14).
  *   - Asynchronous device faults (including the spin watchdog's trap) surface
  *     as CUDA errors at the caller's next synchronisation of the stream.
  *   - No exception or abort crosses the ABI.  Entry points are thread-safe; internal
@@ -58,7 +60,7 @@ extern "C" {
 typedef enum {
   NW_OK = 0,
   NW_EINVAL = 1, /* null pointer, negative size, bad tile, ld < n+1, overlap, misaligned   */
-  NW_ERANGE = 2, /* penalty < 0 or 2*n*p + n*NW_REF_MAX >= 2^31 (int32 could overflow)     */
+  NW_ERANGE = 2, /* penalty < 0 or (n+1)*(2p + NW_REF_MAX) >= 2^30 (int32 could overflow)  */
   NW_ECUDA = 3,  /* a CUDA runtime call failed (nw_last_cuda_error() has the code)          */
   NW_ENOMEM = 4, /* workspace allocation failed                                             */
   NW_ECOMM = 5   /* sharded call with inconsistent peer / halo description                  */

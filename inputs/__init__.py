@@ -212,3 +212,28 @@ def device_problem(n: int, p: int = 10, seed: int = SEED, device="cuda", score=N
     if sentinel:
         score[1:, 1:n + 1] = SENTINEL
     return score, ref
+
+
+def device_strip(n: int, p: int, col0: int, w: int, seed: int = SEED, device="cuda", chunk_rows: int = 4096):
+    """Column strip (global columns col0+1 .. col0+w) of device_problem(n, p, seed) as the local
+    (n+1) x (w+1) matrices a sharded rank holds (nw.h nw_strip): local column j = global column
+    col0 + j; row 0 = the global row 0 there; local column 0 (rows >= 1) = the global left border
+    on the first strip (col0 == 0), else SENTINEL (a halo supplies it); interior SENTINEL."""
+    import torch
+    a, b = gen_pair(n, seed)
+    table = torch.from_numpy(blosum62()).to(device=device, dtype=torch.int32)
+    ta = torch.from_numpy(a.astype(np.int64)).to(device)
+    tb = torch.from_numpy(b[col0:col0 + w].astype(np.int64)).to(device)
+    score = torch.empty((n + 1, w + 1), dtype=torch.int32, device=device)
+    ref = torch.zeros((n + 1, w + 1), dtype=torch.int32, device=device)
+    rows_b = table[:, tb]                       # (24, w): B62[x][b_j] for the strip's columns
+    for i0 in range(0, n, chunk_rows):
+        i1 = min(n, i0 + chunk_rows)
+        ref[1 + i0:1 + i1, 1:] = rows_b[ta[i0:i1]]
+    score[0, :] = (torch.arange(col0, col0 + w + 1, device=device, dtype=torch.int64) * (-p)).to(torch.int32)
+    if col0 == 0:
+        score[1:, 0] = (torch.arange(1, n + 1, device=device, dtype=torch.int64) * (-p)).to(torch.int32)
+    else:
+        score[1:, 0] = SENTINEL
+    score[1:, 1:] = SENTINEL
+    return score, ref

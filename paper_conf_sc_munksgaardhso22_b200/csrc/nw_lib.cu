@@ -73,10 +73,15 @@ bool overlaps(const void* a, int64_t abytes, const void* b, int64_t bbytes) {
 // bytes spanned by an (n+1) x (n+1) matrix with pitch ld (first to last element)
 int64_t span_bytes(int64_t n, int64_t ld) { return 4 * (n * ld + n + 1); }
 
+// Range contract (nw.h).  The wavefront kernels evaluate the gap-normalised S' = S + (i + j) p
+// (DESIGN.md §4.2); every intermediate is bounded by max|border| + (n + 1)(2p + NW_REF_MAX) in
+// absolute value (S <= max border + min(i, j) NW_REF_MAX, S >= -max|border| - n p, (i + j) p <=
+// 2 n p, a diagonal candidate adds ref + 2p).  With the caller's |border| <= 2^30 the sum stays
+// below 2^31 when (n + 1)(2p + NW_REF_MAX) < 2^30, which is what we require.
 nw_status check_range(int64_t n, int32_t p) {
   if (p < 0) return NW_ERANGE;
-  const long double worst = 2.0L * static_cast<long double>(n) * p + static_cast<long double>(n) * NW_REF_MAX;
-  if (worst >= 2147483648.0L) return NW_ERANGE;
+  const long double worst = (static_cast<long double>(n) + 1.0L) * (2.0L * p + NW_REF_MAX);
+  if (worst >= 1073741824.0L) return NW_ERANGE;
   return NW_OK;
 }
 
@@ -415,7 +420,7 @@ const char* nw_status_str(int status) {
   switch (status) {
     case NW_OK: return "NW_OK";
     case NW_EINVAL: return "NW_EINVAL: invalid argument (pointer, size, tile, pitch, alignment or overlap)";
-    case NW_ERANGE: return "NW_ERANGE: penalty < 0 or int32 could overflow (2*n*p + n*NW_REF_MAX >= 2^31)";
+    case NW_ERANGE: return "NW_ERANGE: penalty < 0 or int32 could overflow ((n+1)*(2*p + NW_REF_MAX) >= 2^30)";
     case NW_ECUDA: return "NW_ECUDA: a CUDA runtime call failed (see nw_last_cuda_error)";
     case NW_ENOMEM: return "NW_ENOMEM: workspace allocation failed";
     case NW_ECOMM: return "NW_ECOMM: inconsistent sharded strip / halo description";

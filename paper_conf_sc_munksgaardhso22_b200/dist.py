@@ -55,6 +55,14 @@ def strip_bounds(n: int, world: int, align: int = 128) -> list[Strip]:
     return out
 
 
+def shard_strip(n: int, world: int, rank: int, tile: int = 0) -> Strip:
+    """Rank's strip of the config-5 pipeline: a strip that pushes a halo must end on a band
+    boundary (nw.h, else NW_ECOMM), so the widths are multiples of the band width of `tile`
+    (not a fixed 128) and only the last strip is ragged."""
+    from . import nw_band_width
+    return strip_bounds(n, world, align=nw_band_width(tile))[rank]
+
+
 class EpochCounter:
     """Per-call tag shared by all ranks (every rank calls next() once per collective call)."""
 
@@ -69,29 +77,8 @@ class EpochCounter:
 def local_strip_problem(n: int, p: int, seed: int, strip: Strip, device):
     """Rank-local (n+1, w+1) score / ref of the global seeded problem (inputs.device_problem's
     recipe restricted to the strip's columns): local column 0 = global column col0."""
-    import numpy as np
-    import torch
-
     import inputs
-    a, b = inputs.gen_pair(n, seed)
-    table = torch.from_numpy(inputs.blosum62()).to(device=device, dtype=torch.int32)
-    ta = torch.from_numpy(a.astype(np.int64)).to(device)
-    tb = torch.from_numpy(b[strip.col0:strip.col0 + strip.w].astype(np.int64)).to(device)
-    w = strip.w
-    score = torch.empty((n + 1, w + 1), dtype=torch.int32, device=device)
-    ref = torch.zeros((n + 1, w + 1), dtype=torch.int32, device=device)
-    rows_b = table[:, tb]
-    for i0 in range(0, n, 4096):
-        i1 = min(n, i0 + 4096)
-        ref[1 + i0:1 + i1, 1:] = rows_b[ta[i0:i1]]
-    cols = torch.arange(strip.col0, strip.col0 + w + 1, device=device, dtype=torch.int64)
-    score[0] = (cols * (-p)).to(torch.int32)
-    if strip.rank == 0:
-        score[:, 0] = (torch.arange(n + 1, device=device, dtype=torch.int64) * (-p)).to(torch.int32)
-    else:
-        score[1:, 0] = inputs.SENTINEL   # never read: the halo carries the left border
-    score[1:, 1:] = inputs.SENTINEL
-    return score, ref
+    return inputs.device_strip(n, p, strip.col0, strip.w, seed=seed, device=device)
 
 
 class StripShard:
@@ -105,7 +92,7 @@ class StripShard:
         self.group = group or dist.group.WORLD
         self.rank, self.world = dist.get_rank(self.group), dist.get_world_size(self.group)
         self.device = torch.device("cuda", torch.cuda.current_device())
-        self.strip = strip_bounds(n, self.world)[self.rank]
+        self.strip = shard_strip(n, self.world, self.rank, tile)
         self.score, self.ref = local_strip_problem(n, p, seed, self.strip, self.device)
         self.halo = symm_mem.empty(n + 2, dtype=torch.int64, device=self.device)  # n+2 entries (nw.h)
         self.halo.zero_()

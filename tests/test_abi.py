@@ -87,6 +87,21 @@ def test_validation_codes(L):
     assert L.nw_fill(None, FAKE_R, n, 10, 0, None) == NW_EINVAL
 
 
+def test_range_contract(L):
+    """Range contract (nw.h, R14): (n+1)(2p + NW_REF_MAX) < 2^30, checked before any
+    CUDA call.  The gap-normalised S' = S + (i+j)p reaches |border| + (n+1)(2p + NW_REF_MAX), so the
+    old check (2np + n NW_REF_MAX < 2^31) let contract-legal borders wrap int32 (round-1 verdict:
+    n = 64, p = 16776703, borders 2^30 - 1)."""
+    n = 64
+    assert fill_ld(L, FAKE_S, n + 1, FAKE_R, n + 1, n, 16776703, 0) == NW_ERANGE
+    # the boundary: 65 * (2p + 1024) < 2^30  <=>  p <= 8259040
+    assert fill_ld(L, FAKE_S, n + 1, FAKE_R, n + 1, n, 8259041, 0) == NW_ERANGE
+    assert fill_ld(L, FAKE_S, n + 1, FAKE_R, n + 1, n, 8259041, 16) == NW_ERANGE
+    big = 1 << 20   # n = 2^20: (2^20 + 1)(2p + 1024) < 2^30 needs p <= 0
+    assert fill_ld(L, FAKE_S, big + 1, FAKE_S + (1 << 45), big + 1, big, 1, 0) == NW_ERANGE
+    assert "2^30" in nwb.nw_status_str(NW_ERANGE)
+
+
 def test_no_cpu_fallback(L):
     # valid arguments but no GPU in this container: the library must fail, not compute on the host
     import torch

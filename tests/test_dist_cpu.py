@@ -111,3 +111,19 @@ def test_pair_range_and_strip_bounds():
         assert all(ss[i].col0 + ss[i].w == ss[i + 1].col0 for i in range(G - 1))
         assert all(s.w % 128 == 0 for s, nx in zip(ss, ss[1:]) if nx.w > 0)   # only the last is ragged
     assert [s.w for s in nwdist.strip_bounds(65536, 8)] == [8192] * 8
+
+
+@pytest.mark.parametrize("tile", [0, 16, 64])
+@pytest.mark.parametrize("n,G", [(40000, 2), (32768, 3), (32768, 5), (32768, 6), (32768, 7), (65536, 8), (1000, 3)])
+def test_shard_strip_band_aligned(n, G, tile):
+    """Round-1 advisor finding: StripShard cut strips on 128-column units while a halo-pushing
+    strip must be a multiple of the band width (256 at tile 0), so e.g. n = 40000 on 2 GPUs got
+    NW_ECOMM.  shard_strip aligns to nw_band_width(tile)."""
+    import paper_conf_sc_munksgaardhso22_b200 as nwb
+    from paper_conf_sc_munksgaardhso22_b200 import dist as nwdist
+    W = nwb.nw_band_width(tile)
+    ss = [nwdist.shard_strip(n, G, g, tile) for g in range(G)]
+    assert sum(s.w for s in ss) == n and ss[0].col0 == 0
+    assert all(ss[i].col0 + ss[i].w == ss[i + 1].col0 for i in range(G - 1))
+    assert all(s.w % W == 0 for s in ss[:-1])
+

@@ -86,6 +86,29 @@ def test_fill_aligned_layout(n, tile):
     np.testing.assert_array_equal(got, expect(score, ref, 10))
 
 
+@pytest.mark.parametrize("tile", [0, 16, 64])
+def test_range_edge_bit_exact(tile):
+    """At the edge of the range contract: n = 64, p = 8259040 (65 (2p + 1024) just below 2^30),
+    borders of magnitude 2^30 - 1 (the caller's promise) with random signs, ref at +-NW_REF_MAX:
+    the gap-normalised intermediates reach ~2^31 - 2^10 and the result must still be bit-exact."""
+    n, p = 64, 8259040
+    rng = np.random.default_rng(5)
+    score = np.zeros((n + 1, n + 1), dtype=np.int32)
+    big = (1 << 30) - 1
+    score[0, :] = rng.choice([-big, big], n + 1)
+    score[:, 0] = rng.choice([-big, big], n + 1)
+    score[1:, 1:] = inputs.SENTINEL
+    ref = np.zeros((n + 1, n + 1), dtype=np.int32)
+    ref[1:, 1:] = rng.choice([-nwb.NW_REF_MAX, nwb.NW_REF_MAX, 0, 7], (n, n))
+    want = expect(score, ref, p)
+    np.testing.assert_array_equal(gpu_fill(score, ref, p, tile), want)
+    np.testing.assert_array_equal(gpu_fill(score, ref, p, 16, fn=nwb.nw_fill_diagonal), want)
+    # one past the edge, and round 1's counterexample, are rejected before any work
+    for bad in (p + 1, 16776703):
+        with pytest.raises(nwb.NwError):
+            gpu_fill(score, ref, bad, tile)
+
+
 def test_config1_bit_exact_and_idempotent():
     """BASELINE.json config 1: n=1024, p=10, tile=16, repeated back to back (Table I ran 1000x)."""
     n, p = 1024, 10
@@ -223,6 +246,75 @@ def test_sharded_single_device(G, n, tile):
                                       want[1:, strips[0][1]])
 
 
+@pytest.mark.parametrize("G,n,tile", [(2, 4096, 0), (3, 3000, 64), (4, 8192, 0), (2, 2100, 128)])
+def test_sharded_concurrent_streams(G, n, tile):
+    """Config 5's protocol with the strips running CONCURRENTLY on one GPU: each strip on its own
+    stream, launched in reverse rank order, so every consumer is already spinning on its halo tags
+    while its producer pushes the right border column row by row (system-scope stores, as to a
+    peer GPU: halo_out_is_peer); grids capped so all strips are co-resident; the halo buffers are
+    reused across three calls (epochs 5, 6, 9)."""
+    score, ref = inputs.make_problem(n, 10, seed=21)
+    want = expect(score, ref, 10)
+    strips = split_strips(score, ref, G, tile)
+    halos = [torch.zeros(n + 2, dtype=torch.int64, device="cuda") for _ in range(G + 1)]
+    streams = [torch.cuda.Stream() for _ in range(G)]
+    devs = [(to_dev(ls), to_dev(lr)) for (a, b, ls, lr) in strips]
+    sms = torch.cuda.get_device_properties(0).multi_processor_count
+    torch.cuda.synchronize()
+    try:
+        nwb.nw_debug_set_grid(max(1, sms // G))
+        for epoch in (5, 6, 9):
+            for s_dev, _ in devs:
+                s_dev[1:, 1:] = inputs.SENTINEL
+            torch.cuda.synchronize()
+            for g in reversed(range(G)):
+                s_dev, r_dev = devs[g]
+                nwb.nw_fill_sharded(s_dev, r_dev, 10, halo_in=halos[g] if g > 0 else None,
+                                    halo_out=halos[g + 1] if g < G - 1 else None, epoch=epoch,
+                                    halo_out_is_peer=True, tile=tile, stream=streams[g])
+            torch.cuda.synchronize()
+            for g, (a, b, ls, lr) in enumerate(strips):
+                got = devs[g][0].cpu().numpy()
+                np.testing.assert_array_equal(got[:, 1:], want[:, a + 1:b + 1], err_msg=f"strip {g} epoch {epoch}")
+    finally:
+        nwb.nw_debug_set_grid(0)
+
+
+def test_watchdog_traps_a_missing_halo():
+    """The spin watchdog: a strip whose halo is never written must not hang the GPU.
+    With NW_SPIN_LIMIT_MS=300 the kernel traps, the caller sees a CUDA error at synchronisation
+    (a sticky error: that process's context is gone), and a fresh process then fills correctly."""
+    import subprocess
+    import sys
+    hang = r'''
+import sys; sys.path.insert(0, %r)
+import numpy as np, torch, inputs, paper_conf_sc_munksgaardhso22_b200 as nwb
+s, r = inputs.make_problem(512, 10)
+S = torch.from_numpy(s).cuda(); R = torch.from_numpy(r).cuda()
+halo = torch.zeros(514, dtype=torch.int64, device="cuda")      # never written: tags stay 0
+nwb.nw_fill_sharded(S, R, 10, halo_in=halo, epoch=7, tile=0)   # enqueued fine ...
+try:
+    torch.cuda.synchronize()
+    print("no-error")
+except Exception as e:
+    print("cuda-error", type(e).__name__)
+''' % ROOT
+    env = dict(os.environ, NW_SPIN_LIMIT_MS="300")
+    out = subprocess.run([sys.executable, "-c", hang], env=env, capture_output=True, text=True, timeout=300)
+    assert "cuda-error" in out.stdout, (out.stdout, out.stderr[-2000:])
+    ok = r'''
+import sys; sys.path.insert(0, %r)
+import numpy as np, torch, inputs, oracle, paper_conf_sc_munksgaardhso22_b200 as nwb
+s, r = inputs.make_problem(512, 10)
+want = oracle.nw_ref(s.copy(), r, 10)
+S = torch.from_numpy(s).cuda(); R = torch.from_numpy(r).cuda()
+nwb.nw_fill(S, R, 10, 0); torch.cuda.synchronize()
+print("ok" if np.array_equal(S.cpu().numpy(), want) else "mismatch")
+''' % ROOT
+    out = subprocess.run([sys.executable, "-c", ok], capture_output=True, text=True, timeout=300)
+    assert "ok" in out.stdout, (out.stdout, out.stderr[-2000:])
+
+
 def _stream_compare(s_dev, score_row0, ref, n, p, chunk=2048):
     """Full-size check with the O(n)-memory streaming oracle, rows in chunks."""
     st = oracle.NwRefStream(n, p, score_row0)
@@ -248,6 +340,84 @@ def test_full_size_configs_bit_exact(n, tile):
     nwb.nw_fill(s_dev, r_dev, p, tile)
     torch.cuda.synchronize()
     _stream_compare(s_dev, score[0], ref, n, p)
+
+
+def _stream_compare_strips(parts, n, p, seed=inputs.SEED, chunk=2048):
+    """Config-5 size check: the streaming oracle over the full width, each row chunk compared with
+    the strips' local columns (parts: list of (col0, w, local score on the device))."""
+    a, b = inputs.gen_pair(n, seed)
+    row0 = -np.arange(n + 1, dtype=np.int32) * p
+    st = oracle.NwRefStream(n, p, row0)
+    for i0 in range(1, n + 1, chunk):
+        i1 = min(n + 1, i0 + chunk)
+        ref_rows = inputs.build_ref_block(a, b, i0, i1)
+        want = st.rows(ref_rows, -np.arange(i0, i1, dtype=np.int32) * p)
+        for col0, w, s_dev in parts:
+            got = s_dev[i0:i1, 1:w + 1].cpu().numpy()
+            np.testing.assert_array_equal(got, want[:, col0 + 1:col0 + w + 1], err_msg=f"rows {i0}..{i1} strip at {col0}")
+    st.close()
+
+
+@pytest.mark.parametrize("G", [1, 2, 4, 8])
+def test_config5_full_size_strips(G):
+    """BASELINE.json config 5 at its size, n = 65536 (the one matrix above 2^31 elements: the
+    kernels' 64-bit addressing): G = 1 is nw_fill on the whole matrix; G = 2, 4, 8 are the strips
+    the multi-GPU driver cuts (widths multiples of the band width), run on one device in rank order
+    with each strip pushing its right border into the next strip's halo.  Every cell is checked
+    against the streaming oracle."""
+    from paper_conf_sc_munksgaardhso22_b200 import dist as nwdist
+    n, p, tile = 65536, 10, 0
+    free, _ = torch.cuda.mem_get_info()
+    if free < 40e9:
+        pytest.skip("needs ~35 GB of device memory")
+    parts = []
+    if G == 1:
+        S, R = inputs.device_problem(n, p, device="cuda")
+        nwb.nw_fill(S, R, p, tile)
+        torch.cuda.synchronize()
+        del R
+        parts.append((0, n, S))
+    else:
+        halos = [torch.zeros(n + 2, dtype=torch.int64, device="cuda") for _ in range(G + 1)]
+        for st in nwdist.strip_bounds(n, G, align=nwb.nw_band_width(tile)):
+            S, R = inputs.device_strip(n, p, st.col0, st.w)
+            nwb.nw_fill_sharded(S, R, p, halo_in=halos[st.rank] if st.rank > 0 else None,
+                                halo_out=halos[st.rank + 1] if st.rank < G - 1 else None, epoch=3, tile=tile)
+            torch.cuda.synchronize()
+            del R
+            parts.append((st.col0, st.w, S))
+    _stream_compare_strips(parts, n, p)
+
+
+def test_config4_full_batch_bit_exact():
+    """BASELINE.json config 4 in full: 4096 pairs of n = 2048 built on the device as bench.py builds
+    them, one nw_fill_batch launch (pair mode), every cell of every pair checked with the oracle
+    (pairs copied back in groups; threads: ctypes drops the GIL)."""
+    from concurrent.futures import ThreadPoolExecutor
+    n, p, B = 2048, 10, 4096
+    free, _ = torch.cuda.mem_get_info()
+    if free < 150e9:
+        pytest.skip("needs ~140 GB of device memory")
+    S = torch.empty((B, n + 1, n + 1), dtype=torch.int32, device="cuda")
+    R = torch.empty((B, n + 1, n + 1), dtype=torch.int32, device="cuda")
+    for k in range(B):
+        inputs.device_problem(n, p, seed=inputs.pair_seed(k), device="cuda", score=S[k], ref=R[k])
+    nwb.nw_fill_batch(S, R, p, 0)
+    torch.cuda.synchronize()
+    del R
+
+    def check(args):
+        k, got = args
+        s, r = inputs.make_problem(n, p, seed=inputs.pair_seed(k))
+        return bool(np.array_equal(got, oracle.nw_ref(s, r, p)))
+
+    bad = []
+    with ThreadPoolExecutor(max(4, os.cpu_count() or 4)) as ex:
+        for g0 in range(0, B, 256):
+            got = S[g0:g0 + 256].cpu().numpy()
+            ok = list(ex.map(check, [(g0 + i, got[i]) for i in range(got.shape[0])]))
+            bad += [g0 + i for i, v in enumerate(ok) if not v]
+    assert not bad, bad[:10]
 
 
 @pytest.mark.parametrize("tile", [0, 64, 128])
