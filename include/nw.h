@@ -104,8 +104,8 @@ nw_status nw_fill_batch_ld(int32_t* score, int64_t ld_score, int64_t stride_scor
  *            kernel (entry i = (epoch << 32) | (uint32) score[i][col0], i = 1..n; the kernel
  *            reads entries in 16-byte pairs, hence the spare entry n+1); NULL on rank 0.
  *            Must be zero-filled once before first use; never needs resetting after.
- * halo_out : rank g+1's halo_in (a peer-mapped pointer, e.g. torch symmetric memory) or
- *            NULL on the last rank.  A rank with halo_out needs w % nw_band_width(tile) == 0
+ * halo_out : rank g+1's halo_in (a peer-mapped pointer, e.g. torch symmetric memory, 16-byte
+ *            aligned: entries are stored in 16-byte pairs) or NULL on the last rank.  A rank with halo_out needs w % nw_band_width(tile) == 0
  *            (else NW_ECOMM).  Written with st.relaxed.sys, one entry per row as soon
  *            as the row's last column is final — the NVLink border push is fused into the
  *            wavefront kernel (no host involvement, no separate send/recv).
@@ -216,6 +216,19 @@ nw_status nw_kernel_info(int32_t tile, int32_t device, int64_t* smem_bytes, int3
 /* Test hook: cap the persistent kernel's grid at `grid` CTAs (0 = automatic, #SMs x
  * occupancy).  A 1-CTA grid must still finish (ticket order => deadlock freedom). */
 void nw_debug_set_grid(int32_t grid);
+
+/* Test / experiment switches (process-wide; explicit calls, never environment variables, and none
+ * of them changes a result — only which kernel schedule computes it):
+ *   nw_debug_set_pair_mode(mode): one-band-per-CTA kernels over a batch sweep whole pairs per
+ *     ticket: 0 = automatic (batches of >= 2 pairs per SM), 1 = for any batch of >= 2 pairs,
+ *     -1 = never;
+ *   nw_debug_set_cluster(on): single pairs on the K = 8 kernel as thread-block clusters handing the
+ *     border column over through distributed shared memory (measured slower; off by default);
+ *   nw_debug_set_host_zero_copy(on): nw_fill[_batch]_host runs the kernel directly on pinned host
+ *     buffers (default 1) instead of staging them in device memory. */
+void nw_debug_set_pair_mode(int32_t mode);
+void nw_debug_set_cluster(int32_t on);
+void nw_debug_set_host_zero_copy(int32_t on);
 
 /* Debug hook: persistent-kernel launches record, per task (pair, band) t < cap_tasks, eight
  * uint64 {t, start_ns, end_ns, smid, event_cycles, ref_wait_cycles, border_spin_cycles,

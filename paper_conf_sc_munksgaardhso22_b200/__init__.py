@@ -24,6 +24,7 @@ __all__ = [
     "NwError", "lib", "nw_fill", "nw_fill_batch", "nw_fill_seq", "nw_fill_seq_batch", "nw_fill_sharded", "nw_fill_host", "nw_fill_batch_host",
     "nw_fill_diagonal", "nw_fill_unopt", "nw_traceback", "nw_traceback_batch", "nw_band_width", "nw_launch_count", "nw_diag_lmad",
     "nw_kernel_info", "nw_strip_map", "nw_debug_set_grid", "nw_debug_set_trace", "nw_release_workspace", "nw_status_str",
+    "nw_debug_set_pair_mode", "nw_debug_set_cluster", "nw_debug_set_host_zero_copy",
 ]
 
 NW_OK, NW_EINVAL, NW_ERANGE, NW_ECUDA, NW_ENOMEM, NW_ECOMM = range(6)
@@ -95,6 +96,9 @@ def lib() -> ctypes.CDLL:
             L.nw_debug_set_trace.restype = None
             L.nw_debug_set_grid.argtypes = [_i32]
             L.nw_debug_set_grid.restype = None
+            for f in ("nw_debug_set_pair_mode", "nw_debug_set_cluster", "nw_debug_set_host_zero_copy"):
+                getattr(L, f).argtypes = [_i32]
+                getattr(L, f).restype = None
             L.nw_release_workspace.restype = None
             for f in ("nw_fill", "nw_fill_ld", "nw_fill_batch", "nw_fill_batch_ld", "nw_fill_sharded",
                       "nw_fill_host", "nw_fill_batch_host", "nw_fill_diagonal", "nw_fill_unopt", "nw_kernel_info", "nw_fill_seq",
@@ -346,6 +350,19 @@ def nw_kernel_info(tile: int = 0, device: int = 0):
 
 def nw_debug_set_grid(grid: int):
     lib().nw_debug_set_grid(int(grid))
+
+
+def nw_debug_set_pair_mode(mode: int):
+    """0 automatic, 1 whole pairs per ticket for any batch >= 2, -1 never (nw.h)."""
+    lib().nw_debug_set_pair_mode(int(mode))
+
+
+def nw_debug_set_cluster(on: bool):
+    lib().nw_debug_set_cluster(int(bool(on)))
+
+
+def nw_debug_set_host_zero_copy(on: bool):
+    lib().nw_debug_set_host_zero_copy(int(bool(on)))
 
 
 def nw_debug_set_trace(buf=None):

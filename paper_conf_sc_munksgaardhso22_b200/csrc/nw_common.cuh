@@ -67,8 +67,6 @@ struct StripParams {
   unsigned long long* trace;  // debug: per task 8 x u64 (see nw.h nw_debug_set_trace) or null
   long long trace_cap;
   unsigned long long* trace2;  // debug: per task {store cycles, ref-issue cycles} or null
-  unsigned int dbg_skip;       // timing experiments only (results invalid when nonzero)
-  unsigned int stage_sleep_ns; // staging-warp back-off when idle (NW_STAGE_SLEEP_NS, default below)
   // NEXT-2 (SEQ kernels): ref[i][j] = subst[a[i-1]][b[j-1]] generated on chip
   const uint8_t* seq_a;
   const uint8_t* seq_b;

@@ -122,7 +122,11 @@ cudaError_t setup_wave(int* occ) {
 
 std::mutex g_mu;
 DevInfo g_dev[128];
+// test / experiment switches (explicit API calls, never environment variables: nw.h)
 int g_debug_grid = 0;
+bool g_debug_cluster = false;
+int g_debug_pair_mode = 0;
+bool g_host_zero_copy = true;
 unsigned long long* g_trace = nullptr;
 long long g_trace_cap = 0;
 
@@ -256,22 +260,15 @@ nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* 
   P.ntasks = pairs * nbands;
   const int var = tile_to_variant(tile);
   const int NW = var == 0 ? WCfg8::NW : (var == 1 ? WCfg4::NW : WCfg41::NW);
-  // opt-in (env NW_CLUSTER=1): one pair on the K = 8 kernel as clusters of CL CTAs that hand
-  // the border column over through DSMEM.  Measured slower than the global-memory handoff at
+  // opt-in (nw_debug_set_cluster(1)): one pair on the K = 8 kernel as clusters of CL CTAs that
+  // hand the border column over through DSMEM.  Measured slower than the global-memory handoff at
   // n = 32768 (318 vs 337 GCUPS with CL = 4; CL = 8 clusters do not all fit co-resident).
-  static const bool cluster_env = [] {
-    const char* e = std::getenv("NW_CLUSTER");
-    return e && e[0] == '1';
-  }();
-  const bool use_cluster = var == 0 && !SEQ && pairs == 1 && cluster_env && di->clusters > 0 && g_debug_grid == 0;
+  const bool use_cluster = var == 0 && !SEQ && pairs == 1 && g_debug_cluster && di->clusters > 0 && g_debug_grid == 0;
   P.ngroups = use_cluster ? (P.ntasks + WCfg8C::CL - 1) / WCfg8C::CL : (P.ntasks + NW - 1) / NW;
-  // many independent pairs on a one-band-per-CTA kernel: whole pairs per ticket (pair mode).
-  // NW_PAIR_MODE=0 disables, =2 forces it for any batch (tests)
-  static const int pair_env = [] {
-    const char* e = std::getenv("NW_PAIR_MODE");
-    return e ? static_cast<int>(std::strtol(e, nullptr, 10)) : 1;
-  }();
-  if (!use_cluster && NW == 1 && nbands > 1 && pair_env != 0 && (pair_env == 2 ? pairs > 1 : pairs >= 2LL * di->sms)) {
+  // many independent pairs on a one-band-per-CTA kernel: whole pairs per ticket (pair mode);
+  // nw_debug_set_pair_mode: -1 never, 1 for any batch (tests), 0 automatic
+  if (!use_cluster && NW == 1 && nbands > 1 && g_debug_pair_mode >= 0 &&
+      (g_debug_pair_mode == 1 ? pairs > 1 : pairs >= 2LL * di->sms)) {
     P.pair_mode = 1;
     P.ngroups = pairs;
   }
@@ -284,18 +281,6 @@ nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* 
   P.ticket = w->d_ticket;
   P.err = w->d_err;
   P.spin_limit_ns = spin_limit_ns();
-  {
-    static const unsigned dbg = [] {
-      const char* e = std::getenv("NW_DEBUG_SKIP");
-      return e ? static_cast<unsigned>(std::strtoul(e, nullptr, 0)) : 0u;
-    }();
-    P.dbg_skip = dbg;
-    static const unsigned sleep_ns = [] {
-      const char* e = std::getenv("NW_STAGE_SLEEP_NS");
-      return e ? static_cast<unsigned>(std::strtoul(e, nullptr, 0)) : 0u;
-    }();
-    P.stage_sleep_ns = sleep_ns;
-  }
   P.trace = g_trace;
   P.trace_cap = g_trace_cap;
   P.trace2 = g_trace ? g_trace + 8 * g_trace_cap : nullptr;
@@ -309,7 +294,6 @@ nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* 
   if (use_cluster) {
     const int64_t ncl = std::min<int64_t>(di->clusters, P.ngroups);
     P.ticket_base = w->ticket_next;
-    w->ticket_next += static_cast<unsigned long long>(P.ngroups + ncl);  // every cluster draws one extra ticket
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(static_cast<unsigned>(ncl * WCfg8C::CL));
     cfg.blockDim = dim3(32 * WCfg8C::NWARPS);
@@ -323,6 +307,7 @@ nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* 
     cfg.attrs = at;
     cfg.numAttrs = 1;
     NW_CU(cudaLaunchKernelEx(&cfg, nw_wave_kernel<WCfg8C>, P));
+    w->ticket_next += static_cast<unsigned long long>(P.ngroups + ncl);  // every cluster draws one extra ticket
     return NW_OK;
   }
   const int occ = di->wocc[var][SEQ];
@@ -330,7 +315,6 @@ nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* 
   if (g_debug_grid > 0) grid = g_debug_grid;
   if (grid > P.ngroups) grid = P.ngroups;
   P.ticket_base = w->ticket_next;
-  w->ticket_next += static_cast<unsigned long long>(P.ngroups + grid);  // every CTA draws one extra ticket
   const unsigned g = static_cast<unsigned>(grid);
   if (var == 0 && !SEQ)
     nw_wave_kernel<WCfg8><<<g, 32 * WCfg8::NWARPS, WCfg8::kSmem, st>>>(P);
@@ -345,6 +329,9 @@ nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* 
   else
     nw_wave_kernel<WCfg41S><<<g, 32 * WCfg41S::NWARPS, WCfg41S::kSmem, st>>>(P);
   NW_CU(cudaGetLastError());
+  // only a launched grid consumes tickets (every CTA draws one past the last group): a failed
+  // launch leaves the device counter and the host base in step
+  w->ticket_next += static_cast<unsigned long long>(P.ngroups + grid);
   return NW_OK;
 }
 
@@ -411,6 +398,9 @@ struct HostBufs {
   cudaStream_t st = nullptr;
 };
 HostBufs g_host[128];
+// one staged host call per device at a time: the staging buffers and their stream are per device
+// (the lock spans the reallocation, the copies, the launch and the final synchronisation)
+std::mutex g_host_mu[128];
 
 }  // namespace
 
@@ -476,7 +466,7 @@ nw_status nw_fill_sharded(const nw_strip* sp, int32_t penalty, int32_t tile, voi
   if (overlaps(S.score, 4 * (S.n * S.ld_score + S.w + 1), S.ref, 4 * (S.n * S.ld_ref + S.w + 1))) return NW_EINVAL;
   if ((S.halo_in || S.halo_out) && S.epoch == 0) return NW_ECOMM;
   if ((S.halo_in && (reinterpret_cast<uintptr_t>(S.halo_in) & 15)) ||
-      (S.halo_out && (reinterpret_cast<uintptr_t>(S.halo_out) & 7)))
+      (S.halo_out && (reinterpret_cast<uintptr_t>(S.halo_out) & 15)))
     return NW_ECOMM;
   // a strip that pushes a halo must end on a band boundary (its last band is then full width)
   if (S.halo_out && S.w % nw_band_width(tile) != 0) return NW_ECOMM;
@@ -528,11 +518,7 @@ nw_status nw_fill_batch_host(int32_t* score_host, const int32_t* ref_host, int64
   // Pinned (device-mapped) host buffers: the kernel streams ref in and score out over the host
   // link itself (zero copy, both directions at once, overlapped with the wavefront) instead of
   // copy-in / compute / copy-out.  Pageable buffers take the staged path below.
-  static const bool zero_copy = [] {
-    const char* e = std::getenv("NW_HOST_ZEROCOPY");
-    return !(e && e[0] == '0');
-  }();
-  if (zero_copy) {
+  if (g_host_zero_copy) {
     cudaPointerAttributes as{}, ar{};
     const bool ok = cudaPointerGetAttributes(&as, score_host) == cudaSuccess &&
                     cudaPointerGetAttributes(&ar, ref_host) == cudaSuccess && as.type == cudaMemoryTypeHost &&
@@ -547,6 +533,7 @@ nw_status nw_fill_batch_host(int32_t* score_host, const int32_t* ref_host, int64
       return NW_OK;
     }
   }
+  std::lock_guard<std::mutex> hlk(g_host_mu[device]);
   {
     std::lock_guard<std::mutex> lk(g_mu);
     if (elems > hb.elems) {
@@ -695,6 +682,9 @@ int32_t nw_strip_map(int64_t n, int64_t width, int32_t tile, int32_t band, int32
 }
 
 void nw_debug_set_grid(int32_t grid) { g_debug_grid = grid > 0 ? grid : 0; }
+void nw_debug_set_pair_mode(int32_t mode) { g_debug_pair_mode = mode < 0 ? -1 : (mode > 0 ? 1 : 0); }
+void nw_debug_set_cluster(int32_t on) { g_debug_cluster = on != 0; }
+void nw_debug_set_host_zero_copy(int32_t on) { g_host_zero_copy = on != 0; }
 
 void nw_debug_set_trace(uint64_t* dev_buf, int64_t cap_tasks) {
   std::lock_guard<std::mutex> lk(g_mu);

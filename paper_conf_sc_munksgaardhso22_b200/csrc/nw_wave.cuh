@@ -65,6 +65,16 @@ namespace nwb200 {
 #ifndef NW_PF_AT
 #define NW_PF_AT 8
 #endif
+// Experiment builds only (scripts/, _build.build_variant): NW_DEBUG_SKIP skips parts of the
+// staging (bits 0-3: results invalid), relaxes the progress words (bit 4) or switches the L2
+// prefetch to bulk prefetches (bit 5); NW_STAGE_SLEEP_NS backs idle staging warps off.  Both are
+// compile-time: the shipped library has neither (a run-time switch could silently corrupt results).
+#ifndef NW_DEBUG_SKIP
+#define NW_DEBUG_SKIP 0u
+#endif
+#ifndef NW_STAGE_SLEEP_NS
+#define NW_STAGE_SLEEP_NS 0
+#endif
 // CL > 1: thread-block clusters of CL CTAs (one band each, NW = 1) take CL consecutive bands;
 // inside a cluster the border column goes straight into the next CTA's shared memory (DSMEM).
 template <int K_, bool SEQ_, int NW_, int SPB_, int CL_ = 1>
@@ -159,42 +169,33 @@ template <int OFF>
 __device__ __forceinline__ void sts128_ring(uint32_t a, int x, int y, int z, int w) {
   asm volatile("st.shared.v4.b32 [%0+%5], {%1, %2, %3, %4};" ::"r"(a), "r"(x), "r"(y), "r"(z), "r"(w), "n"(OFF));
 }
-// border-entry stores {value, tag}: v2.b32 straight from the value register (a 64-bit temporary
-// register pair reused step after step made every store wait for the previous one's operand read)
-__device__ __forceinline__ void st_entry_gpu_p(bool pred, uint64_t* p, uint32_t lo, uint32_t hi) {
-  asm volatile("{ .reg .pred q; setp.ne.b32 q, %0, 0; @q st.relaxed.gpu.global.v2.b32 [%1], {%2, %3}; }" ::"r"(static_cast<int>(pred)),
-               "l"(p), "r"(lo), "r"(hi)
-               : "memory");
-}
-__device__ __forceinline__ void st_entry_sys_p(bool pred, uint64_t* p, uint32_t lo, uint32_t hi) {
-  asm volatile("{ .reg .pred q; setp.ne.b32 q, %0, 0; @q st.relaxed.sys.global.v2.b32 [%1], {%2, %3}; }" ::"r"(static_cast<int>(pred)),
-               "l"(p), "r"(lo), "r"(hi)
-               : "memory");
-}
-__device__ __forceinline__ void st_entry_smem_p(bool pred, uint32_t a, uint32_t lo, uint32_t hi) {
-  asm volatile("{ .reg .pred q; setp.ne.b32 q, %0, 0; @q st.volatile.shared.v2.b32 [%1], {%2, %3}; }" ::"r"(static_cast<int>(pred)),
-               "r"(a), "r"(lo), "r"(hi)
-               : "memory");
-}
+// Border-entry stores {value, tag}.  Every entry is ONE 8-byte element (a .b64 scalar or an element
+// of a .v2.b64 vector), so a relaxed load that sees an entry's tag sees the value stored with it
+// (single-copy atomicity of aligned 8-byte elements; PTX treats a vector access as accesses to its
+// elements).  The two 32-bit halves are packed into the 64-bit operand inside the asm block.
+#define NW_ENT1(SCOPE_SPACE, ADDR_T)                                                                         \
+  asm volatile("{ .reg .pred q; .reg .b64 e; setp.ne.b32 q, %0, 0; mov.b64 e, {%2, %3}; @q st." SCOPE_SPACE \
+               ".b64 [%1], e; }" ::"r"(static_cast<int>(pred)),                                              \
+               ADDR_T(p), "r"(lo), "r"(hi)                                                                   \
+               : "memory")
+#define NW_ENT2(SCOPE_SPACE, ADDR_T)                                                                          \
+  asm volatile("{ .reg .pred q; .reg .b64 e0, e1; setp.ne.b32 q, %0, 0; mov.b64 e0, {%2, %3}; mov.b64 e1, {%4, %5}; " \
+               "@q st." SCOPE_SPACE ".v2.b64 [%1], {e0, e1}; }" ::"r"(static_cast<int>(pred)),                \
+               ADDR_T(p), "r"(v0), "r"(t0), "r"(v1), "r"(t1)                                                  \
+               : "memory")
+__device__ __forceinline__ void st_entry_gpu_p(bool pred, uint64_t* p, uint32_t lo, uint32_t hi) { NW_ENT1("relaxed.gpu.global", "l"); }
+__device__ __forceinline__ void st_entry_sys_p(bool pred, uint64_t* p, uint32_t lo, uint32_t hi) { NW_ENT1("relaxed.sys.global", "l"); }
+__device__ __forceinline__ void st_entry_smem_p(bool pred, uint32_t p, uint32_t lo, uint32_t hi) { NW_ENT1("volatile.shared", "r"); }
 
-// two consecutive border entries (rows 2k, 2k+1: 16-byte aligned) in one v4 store
+// two consecutive border entries (rows 2k, 2k+1: 16-byte aligned) in one store of two 8-byte elements
 __device__ __forceinline__ void st_pair_gpu_p(bool pred, uint64_t* p, uint32_t v0, uint32_t t0, uint32_t v1, uint32_t t1) {
-  asm volatile("{ .reg .pred q; setp.ne.b32 q, %0, 0; @q st.relaxed.gpu.global.v4.b32 [%1], {%2, %3, %4, %5}; }" ::"r"(
-                   static_cast<int>(pred)),
-               "l"(p), "r"(v0), "r"(t0), "r"(v1), "r"(t1)
-               : "memory");
+  NW_ENT2("relaxed.gpu.global", "l");
 }
 __device__ __forceinline__ void st_pair_sys_p(bool pred, uint64_t* p, uint32_t v0, uint32_t t0, uint32_t v1, uint32_t t1) {
-  asm volatile("{ .reg .pred q; setp.ne.b32 q, %0, 0; @q st.relaxed.sys.global.v4.b32 [%1], {%2, %3, %4, %5}; }" ::"r"(
-                   static_cast<int>(pred)),
-               "l"(p), "r"(v0), "r"(t0), "r"(v1), "r"(t1)
-               : "memory");
+  NW_ENT2("relaxed.sys.global", "l");
 }
-__device__ __forceinline__ void st_pair_smem_p(bool pred, uint32_t a, uint32_t v0, uint32_t t0, uint32_t v1, uint32_t t1) {
-  asm volatile("{ .reg .pred q; setp.ne.b32 q, %0, 0; @q st.volatile.shared.v4.b32 [%1], {%2, %3, %4, %5}; }" ::"r"(
-                   static_cast<int>(pred)),
-               "r"(a), "r"(v0), "r"(t0), "r"(v1), "r"(t1)
-               : "memory");
+__device__ __forceinline__ void st_pair_smem_p(bool pred, uint32_t p, uint32_t v0, uint32_t t0, uint32_t v1, uint32_t t1) {
+  NW_ENT2("volatile.shared", "r");
 }
 
 // DSMEM (shared::cluster addresses from mapa): the next CTA's incoming ring / progress word
@@ -203,17 +204,11 @@ __device__ __forceinline__ uint32_t mapa_u32(uint32_t a, uint32_t rank) {
   asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(d) : "r"(a), "r"(rank));
   return d;
 }
-__device__ __forceinline__ void st_pair_dsmem_p(bool pred, uint32_t a, uint32_t v0, uint32_t t0, uint32_t v1, uint32_t t1) {
-  asm volatile("{ .reg .pred q; setp.ne.b32 q, %0, 0; @q st.relaxed.cluster.shared::cluster.v4.b32 [%1], {%2, %3, %4, %5}; }" ::"r"(
-                   static_cast<int>(pred)),
-               "r"(a), "r"(v0), "r"(t0), "r"(v1), "r"(t1)
-               : "memory");
+__device__ __forceinline__ void st_pair_dsmem_p(bool pred, uint32_t p, uint32_t v0, uint32_t t0, uint32_t v1, uint32_t t1) {
+  NW_ENT2("relaxed.cluster.shared::cluster", "r");
 }
-__device__ __forceinline__ void st_entry_dsmem_p(bool pred, uint32_t a, uint32_t lo, uint32_t hi) {
-  asm volatile("{ .reg .pred q; setp.ne.b32 q, %0, 0; @q st.relaxed.cluster.shared::cluster.v2.b32 [%1], {%2, %3}; }" ::"r"(
-                   static_cast<int>(pred)),
-               "r"(a), "r"(lo), "r"(hi)
-               : "memory");
+__device__ __forceinline__ void st_entry_dsmem_p(bool pred, uint32_t p, uint32_t lo, uint32_t hi) {
+  NW_ENT1("relaxed.cluster.shared::cluster", "r");
 }
 __device__ __forceinline__ int ld_dsmem_b32(uint32_t a) {
   int v;
@@ -297,7 +292,9 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
   for (int i = 0; i < K; ++i) wmask |= static_cast<uint32_t>(32 * i + t < g.ws) << i;
   const uint64_t ldr4 = 4ull * static_cast<uint64_t>(P.ldr), lds4 = 4ull * static_cast<uint64_t>(P.lds);
   const uint64_t gR0 = SEQ ? 0ull : reinterpret_cast<uint64_t>(g.Rf + g.c0 + t);  // (row 0, word t) of the ref segment
-  const bool strict = (P.dbg_skip & 16u) != 0;  // (experiments: release-fenced progress stores)
+  // progress words: release stores / acquire loads (NW_DEBUG_SKIP bit 4, experiment builds: relaxed;
+  // measured: no difference, 3.08 vs 3.11 ms at n = 32768, 37.65 vs 37.53 ms on config 4)
+  constexpr bool strict = (NW_DEBUG_SKIP & 16u) == 0;
   const uint64_t gS0 = reinterpret_cast<uint64_t>(g.S + g.c0 + t);
   int consumed = 0, complete = 0;  // cached compute-warp progress
   int landed = 0, stored = 0;      // published to the compute warp
@@ -330,11 +327,11 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
     }
   };
   // L2 prefetch of chunk k's rows: CH rows x NL 128-byte lines, lane t handles lines t, t+32, ...
-  // (P.dbg_skip bit 5: one cp.async.bulk.prefetch.L2 per row instead)
+  // (NW_DEBUG_SKIP bit 5, experiment builds: one cp.async.bulk.prefetch.L2 per row instead)
   const uint32_t pf_bytes = static_cast<uint32_t>((4 * g.ws + 12 + 15) & ~15);
   auto prefetch_chunk = [&](int k) {
     if constexpr (!SEQ) {
-      if (P.dbg_skip & 32u) {
+      if constexpr ((NW_DEBUG_SKIP & 32u) != 0) {
         const int rp = CH * k + 1 + t;
         if (t < CH && rp <= n) {
           const uint64_t ga = (reinterpret_cast<uint64_t>(g.Rf + g.c0) + static_cast<uint64_t>(static_cast<long long>(rp)) * ldr4) & ~15ull;
@@ -415,7 +412,7 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
       const int need = CH * kr + CH - RR;
       if (consumed < need) prog_read(from_c, consumed, complete);
       if (consumed >= need) {
-        if (!(P.dbg_skip & 5u)) issue_chunk(kr);  // (timing experiments only: results invalid)
+        if constexpr (!(NW_DEBUG_SKIP & 5u)) issue_chunk(kr);  // (experiment builds only: results invalid)
         if (kr + C::PFC < nch) prefetch_chunk(kr + C::PFC);
         cp_async_commit();
         ++kr;
@@ -427,7 +424,7 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
       if (complete < need) prog_read(from_c, consumed, complete);
       if (complete >= need) {
         const long long cs0 = tracing ? clock64() : 0;
-        if (!(P.dbg_skip & 9u)) store_chunk(ks);
+        if constexpr (!(NW_DEBUG_SKIP & 9u)) store_chunk(ks);
         if (tracing) st_busy += clock64() - cs0, st_gap_sum += cs0 - st_last, st_last = clock64();
         ks += kstep;
         did = true;
@@ -445,8 +442,8 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
       }
       if (nl > landed) {
         landed = nl;
-        // relaxed (no MEMBAR): every lane's copies have completed (wait_group) before the
-        // __syncwarp and this store; a fence here would also wait for nothing useful
+        // release: every lane's copies have completed (wait_group) before the __syncwarp and
+        // this store; the compute warp's acquire load orders its ring reads after them
         prog_publish(to_ref, landed, 0, !strict);
       }
       done = landed == n;
@@ -455,9 +452,8 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
       const int ns = min(ks, nch);  // my chunks below ns are stored
       if (ns > stored) {
         stored = ns;
-        // relaxed: what the compute warp needs is that the ring slots were READ, and every STG
-        // above consumed its LDS result before this store issues (a release fence would wait
-        // for the global stores to be acknowledged: ~130 cycles of compute-warp stall per event)
+        // release: the ring slots were READ (every STG above consumed its LDS result) before the
+        // compute warp, after its acquire load, rewrites them
         prog_publish(to_st, stored, 0, !strict);
       }
       done = done && ks >= nch;
@@ -468,7 +464,7 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
     } else {
       // idle: back off (a tight poll of the progress words competes with the compute warp's
       // shared-memory / shuffle traffic in the SM's MIO pipe)
-      if (P.stage_sleep_ns) __nanosleep(P.stage_sleep_ns);
+      if constexpr (NW_STAGE_SLEEP_NS > 0) __nanosleep(NW_STAGE_SLEEP_NS);
       if ((++idle & 255u) == 0) {
         const uint64_t now = globaltimer_ns();
         if (idle == 256) tw = now;
@@ -502,7 +498,7 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
   const unsigned long long t_task0 = tracing ? globaltimer_ns() : 0ull;
   long long spin_cyc = 0, wait_cyc = 0, bp_cyc = 0, steady_cyc = 0, steady_blocks = 0;
   long long ph_cyc[3] = {0, 0, 0}, st_wait_cyc = 0, pub_cyc = 0;  // event phases: publish + staging wait, border (+ spin), back-pressure + misc
-  const bool strict = (P.dbg_skip & 16u) != 0;  // (experiments: release-fenced progress stores)
+  constexpr bool strict = (NW_DEBUG_SKIP & 16u) == 0;  // release-stored progress words (above)
 
   const BandGeo<C> g(P, task, wsm);
   const int n = g.n, p = g.p, band = g.band, c0 = g.c0, ws = g.ws;
@@ -790,9 +786,8 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     // ---- event Q.  To the staging warp: ref rows <= sig0-30 consumed (lane 31 read row sig0-30
     // at step sig0-1), score rows <= sig0-31 complete (lane 31 wrote row sig0-31 at step sig0-1).
     const long long ce0 = tracing ? clock64() : 0;
-    // relaxed: the warp's earlier shared-memory accesses are performed in order before this
-    // store (__syncwarp, then one lane's store; the MIO processes a warp's shared-memory
-    // instructions in order) -- a release fence here cost ~200 cycles per event (MEMBAR.CTA)
+    // release after __syncwarp: every lane's ring writes (score) and reads (ref) of the earlier
+    // steps happen before the staging warps' acquire of this word
     prog_publish(to_s, max(0, sig0 - 30), max(0, sig0 - 31), !strict);
     if (tracing) pub_cyc += clock64() - ce0;
     {
@@ -980,7 +975,7 @@ __global__ void __launch_bounds__(32 * C::NWARPS, 1) nw_wave_kernel(const __grid
       __syncthreads();
       group = static_cast<long long>(*s_group - P.ticket_base);
     }
-    if (group >= P.ngroups) break;
+    if (group < 0 || group >= P.ngroups) break;  // (< 0: a stale ticket base; never draw a negative task)
     // pair mode (many independent pairs, NW = 1): a ticket is a whole pair and the CTA sweeps its
     // bands one after the other -- band k's border column is already complete when it starts
     // (no band-to-band pipeline fill, no polling)

@@ -121,6 +121,25 @@ def test_config1_bit_exact_and_idempotent():
     np.testing.assert_array_equal(s.cpu().numpy(), want)
 
 
+@pytest.mark.parametrize("tile", [0, 16, 64])
+def test_flag_race_stress_1000(tile):
+    """The band-to-band handoff under repetition (Table I ran 1000 times):
+    n = 1024, 1000 launches, each on a sentinel-reset interior and each compared on the device
+    with the oracle's matrix (a stale or torn border entry would show as a wrong cell)."""
+    n, p = 1024, 10
+    score, ref = inputs.make_problem(n, p, seed=1000 + tile)
+    want = torch.from_numpy(expect(score, ref, p)).cuda()
+    s, r = to_dev(score), to_dev(ref)
+    bad = []
+    for rep in range(1000):
+        s[1:, 1:] = inputs.SENTINEL
+        nwb.nw_fill(s, r, p, tile)
+        if not torch.equal(s, want):
+            bad.append(rep)
+    torch.cuda.synchronize()
+    assert not bad, bad[:10]
+
+
 @pytest.mark.parametrize("grid", [1, 3])
 def test_small_grids_deadlock_free(grid):
     """Ticket order => a CTA only waits on bands held by running CTAs: a 1-CTA grid must finish."""
@@ -477,50 +496,37 @@ def test_config4_shape_batch_bit_exact():
     assert all(ok), [k for k, v in enumerate(ok) if not v][:10]
 
 
-@pytest.mark.gpu
 def test_cluster_dsmem_handoff_opt_in():
-    """NW_CLUSTER=1 (opt-in): single pairs run as clusters of 4 CTAs whose border columns pass
-    through distributed shared memory; bit-exact against the oracle (subprocess: the switch is
-    read once per process)."""
-    import subprocess
-    import sys
-    code = r'''
-import sys; sys.path.insert(0, %r)
-import numpy as np, torch, inputs, oracle, paper_conf_sc_munksgaardhso22_b200 as nwb
-for n in (1, 255, 256, 1000, 1024, 3000):
-    s, r = inputs.make_problem(n, 10)
-    want = oracle.nw_ref(s.copy(), r, 10)
-    S = torch.from_numpy(s).cuda(); R = torch.from_numpy(r).cuda()
-    nwb.nw_fill(S, R, 10, 0); torch.cuda.synchronize()
-    assert np.array_equal(S.cpu().numpy(), want), n
-print("ok")
-''' % ROOT
-    env = dict(os.environ, NW_CLUSTER="1")
-    out = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=600)
-    assert out.returncode == 0 and "ok" in out.stdout, out.stderr[-2000:]
+    """nw_debug_set_cluster(1) (opt-in): single pairs run as clusters of 4 CTAs whose border
+    columns pass through distributed shared memory; bit-exact against the oracle."""
+    try:
+        nwb.nw_debug_set_cluster(True)
+        for n in (1, 255, 256, 1000, 1024, 3000):
+            s, r = inputs.make_problem(n, 10)
+            np.testing.assert_array_equal(gpu_fill(s, r, 10, 0), expect(s, r, 10), err_msg=str(n))
+    finally:
+        nwb.nw_debug_set_cluster(False)
 
 
-@pytest.mark.gpu
 def test_pair_mode_batches_forced():
     """Pair mode (a CTA sweeps all bands of a pair in turn; automatic for large batches) forced
-    on small ragged batches with NW_PAIR_MODE=2, both one-band-per-CTA kernels (tiles 0, 64)."""
-    import subprocess
-    import sys
-    code = r'''
-import sys; sys.path.insert(0, %r)
-import numpy as np, torch, inputs, oracle, paper_conf_sc_munksgaardhso22_b200 as nwb
-for B, n, tile in ((3, 700, 0), (5, 257, 64), (2, 1024, 0), (4, 1500, 64), (3, 100, 0)):
-    ss, rs, want = [], [], []
-    for k in range(B):
-        s, r = inputs.make_problem(n, 10, seed=inputs.pair_seed(k))
-        ss.append(s); rs.append(r); want.append(oracle.nw_ref(s.copy(), r, 10))
-    S = torch.from_numpy(np.stack(ss)).cuda(); R = torch.from_numpy(np.stack(rs)).cuda()
-    nwb.nw_fill_batch(S, R, 10, tile); torch.cuda.synchronize()
-    got = S.cpu().numpy()
-    for k in range(B):
-        assert np.array_equal(got[k], want[k]), (B, n, tile, k)
-print("ok")
-''' % ROOT
-    env = dict(os.environ, NW_PAIR_MODE="2")
-    out = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=600)
-    assert out.returncode == 0 and "ok" in out.stdout, out.stderr[-2000:]
+    on small ragged batches (nw_debug_set_pair_mode(1)), both one-band-per-CTA kernels (tiles 0,
+    64); and switched off (-1) for a batch large enough to enable it automatically."""
+    try:
+        for mode, cases in ((1, ((3, 700, 0), (5, 257, 64), (2, 1024, 0), (4, 1500, 64), (3, 100, 0))),
+                            (-1, ((600, 64, 0),))):
+            nwb.nw_debug_set_pair_mode(mode)
+            for B, n, tile in cases:
+                ss, rs, want = [], [], []
+                for k in range(B):
+                    s, r = inputs.make_problem(n, 10, seed=inputs.pair_seed(k))
+                    ss.append(s), rs.append(r), want.append(expect(s, r, 10))
+                S = torch.from_numpy(np.stack(ss)).cuda()
+                R = torch.from_numpy(np.stack(rs)).cuda()
+                nwb.nw_fill_batch(S, R, 10, tile)
+                torch.cuda.synchronize()
+                got = S.cpu().numpy()
+                for k in range(B):
+                    np.testing.assert_array_equal(got[k], want[k], err_msg=f"{mode} {B} {n} {tile} {k}")
+    finally:
+        nwb.nw_debug_set_pair_mode(0)
