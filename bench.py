@@ -105,8 +105,45 @@ def ncu_traffic(workload, tile):
         return None
 
 
-def cpu_baseline(cfg, gpu_last_row=None):
-    """The oracle as it stands (single-threaded C) on a bounded sample of the workload."""
+# Cycles of one wavefront step of one band in isolation (a warp per SM sub-partition, no staging
+# stalls), measured on B200 with scripts/ubench_mw.cu (round 2): K = 8: 88.1; K = 4 one band per
+# SM: 53.1; K = 4 two bands per SM: 52.2 (each).
+STEP_CYCLES = {8: 88.1, 4: 53.1}
+
+
+def latency_floor(n, B, tile, nwb, kern_ms, clocks, variant, world, strips):
+    """The other roofline of the wavefront: its critical path.  A band's warp needs n + 31 steps
+    (its 32 lanes are skewed by one row) and band k+1 can start no earlier than 32 steps after band
+    k, so one pair takes at least n + 31 * nbands steps; in pair mode (large batches) a CTA sweeps
+    its pairs' bands back to back: ceil(pairs / CTAs) * nbands * (n + 31) steps.  frac = that floor
+    at the isolated step time / the measured kernel time."""
+    if variant not in ("strip", "seq") or strips:
+        return None
+    W = nwb.nw_band_width(tile)
+    K = W // 32
+    nb = -(-n // W)
+    c = STEP_CYCLES[K]
+    mhz = clocks.get("sm_mhz") or 1965.0
+    if B == 1:
+        steps = n + 31 * nb
+        how = f"n + 31 * nbands = {n} + 31 * {nb}"
+    else:
+        ki = nwb.nw_kernel_info(tile)
+        grid = ki["ctas_per_sm"] * ki["num_sms"]
+        per = -(-(B // world) // grid)
+        steps = per * nb * (n + 31)
+        how = f"ceil(pairs / {grid} CTAs) * nbands * (n + 31) = {per} * {nb} * {n + 31}"
+    floor_ms = steps * c / (mhz * 1e3)
+    return {"bound": "wavefront critical path", "critical_steps": steps, "steps_formula": how,
+            "step_cycles_isolated": c, "step_cycles_source": "scripts/ubench_mw.cu (B200, round 2)",
+            "sm_mhz": mhz, "floor_ms": floor_ms, "frac": floor_ms / kern_ms,
+            "cycles_per_critical_step": kern_ms * mhz * 1e3 / steps}
+
+
+def cpu_baseline(cfg, gpu_score=None):
+    """The oracle as it stands (single-threaded C) on a bounded sample of the workload; when the
+    GPU's result is given (device tensor), every oracle row / pair is compared with it (outside the
+    oracle's timing)."""
     import numpy as np
 
     import inputs
@@ -120,39 +157,41 @@ def cpu_baseline(cfg, gpu_last_row=None):
         t_or = 0.0
         rows_done = 0
         budget = float(os.environ.get("NW_CPU_BASELINE_S", "25"))
-        last = None
+        exact = None if gpu_score is None else True
         for i0 in range(1, n + 1, 1024):
             i1 = min(n + 1, i0 + 1024)
             blk = inputs.build_ref_block(a, b, i0, i1)
             col0 = (-np.arange(i0, i1, dtype=np.int64) * p).astype(np.int32)
             t = time.perf_counter()
-            out = st.rows(blk, col0, want_out=(i1 == n + 1))
+            out = st.rows(blk, col0, want_out=True)  # (the oracle produces the rows; timed either way)
             t_or += time.perf_counter() - t
             rows_done = i1 - 1
-            if i1 == n + 1:
-                last = out[-1]
+            if gpu_score is not None:
+                exact = exact and bool(np.array_equal(out, gpu_score[i0:i1, : n + 1].cpu().numpy()))
             if t_or > budget:
                 break
         st.close()
         cells = rows_done * n
         sample = f"rows 1..{rows_done} of the n={n} matrix (streaming oracle, {cells:.3e} cells)"
-        exact = None
-        if last is not None and gpu_last_row is not None:
-            exact = bool(np.array_equal(last, gpu_last_row))
         return {"value": cells / t_or / 1e9, "unit": "GCUPS", "cores": 1, "kind": "oracle",
-                "sample": sample, "seconds": t_or, "last_row_bit_exact": exact}
+                "sample": sample, "seconds": t_or, "bit_exact_rows": rows_done if exact else None,
+                "bit_exact": exact}
     # batch: the first pairs of the batch, one by one
     t_or, cells, k = 0.0, 0, 0
+    exact = None if gpu_score is None else True
     budget = float(os.environ.get("NW_CPU_BASELINE_S", "15"))
     while t_or < budget and k < cfg["batch"]:
         s, r = inputs.make_problem(n, p, seed=inputs.pair_seed(k))
         t = time.perf_counter()
-        oracle.nw_ref(s, r, p)
+        want = oracle.nw_ref(s, r, p)
         t_or += time.perf_counter() - t
+        if gpu_score is not None:
+            exact = exact and bool(np.array_equal(want, gpu_score[k].cpu().numpy()))
         cells += n * n
         k += 1
     return {"value": cells / t_or / 1e9, "unit": "GCUPS", "cores": 1, "kind": "oracle",
-            "sample": f"first {k} of {cfg['batch']} pairs (n={n})", "seconds": t_or}
+            "sample": f"first {k} of {cfg['batch']} pairs (n={n})", "seconds": t_or,
+            "bit_exact_pairs": k if exact else None, "bit_exact": exact}
 
 
 def run_reference(args, cfg, rank):
@@ -305,6 +344,8 @@ def main():
             if args.variant in ("strip", "seq")
             else f"nw_diag_kernel<{tile}> x{nwb.nw_launch_count(1, n, tile)} launches (+copies: unopt)",
             "kernel_ms_mean": kern_ms, "kernel_ms_median": statistics.median(per_launch)}
+    roof["latency"] = latency_floor(n, B if not strips else 1, tile, nwb, kern_ms, clk.summary(), args.variant,
+                                    world, strips)
     out = {"metric": METRIC, "value": value, "unit": "GCUPS", "n_gpus": world, "steps": args.steps,
            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
            "scaling": "strong" if world > 1 else "weak", "vs_baseline": None, "dtype": "int32",
@@ -389,9 +430,10 @@ def main():
         out["gpu_launches_e2e"] = args.e2e_steps + 1
         nwb.nw_release_workspace()
         del hr, hs
-    gpu_last = S[n].cpu().numpy() if B == 1 and not strips else None
     if rank == 0 and not args.no_cpu:
-        out["cpu_baseline"] = cpu_baseline(cfg, gpu_last)
+        # (strips: the local strip is not the whole matrix; batch: this rank's first pairs are the
+        # global pairs lo.. -- rank 0 holds the first)
+        out["cpu_baseline"] = cpu_baseline(cfg, S if not strips else None)
     if rank == 0:
         print(json.dumps(out), flush=True)
     if world > 1:

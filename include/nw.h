@@ -61,9 +61,10 @@ typedef enum {
   NW_OK = 0,
   NW_EINVAL = 1, /* null pointer, negative size, bad tile, ld < n+1, overlap, misaligned   */
   NW_ERANGE = 2, /* penalty < 0 or (n+1)*(2p + NW_REF_MAX) >= 2^30 (int32 could overflow)  */
-  NW_ECUDA = 3,  /* a CUDA runtime call failed (nw_last_cuda_error() has the code)          */
-  NW_ENOMEM = 4, /* workspace allocation failed                                             */
-  NW_ECOMM = 5   /* sharded call with inconsistent peer / halo description                  */
+  NW_ECUDA = 3,  /* a CUDA runtime call failed, including a workspace allocation            */
+                 /* (nw_last_cuda_error() has the code)                                     */
+  NW_ECOMM = 4   /* sharded call with inconsistent peer / halo description                  */
+  /* (the numbering is SURVEY.md §8(b)'s) */
 } nw_status;
 
 const char* nw_status_str(int status);

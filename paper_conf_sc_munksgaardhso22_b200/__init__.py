@@ -27,7 +27,7 @@ __all__ = [
     "nw_debug_set_pair_mode", "nw_debug_set_cluster", "nw_debug_set_host_zero_copy",
 ]
 
-NW_OK, NW_EINVAL, NW_ERANGE, NW_ECUDA, NW_ENOMEM, NW_ECOMM = range(6)
+NW_OK, NW_EINVAL, NW_ERANGE, NW_ECUDA, NW_ECOMM = range(5)  # SURVEY.md §8(b) numbering
 NW_REF_MAX = 1024
 
 _lock = threading.Lock()

@@ -411,8 +411,7 @@ const char* nw_status_str(int status) {
     case NW_OK: return "NW_OK";
     case NW_EINVAL: return "NW_EINVAL: invalid argument (pointer, size, tile, pitch, alignment or overlap)";
     case NW_ERANGE: return "NW_ERANGE: penalty < 0 or int32 could overflow ((n+1)*(2*p + NW_REF_MAX) >= 2^30)";
-    case NW_ECUDA: return "NW_ECUDA: a CUDA runtime call failed (see nw_last_cuda_error)";
-    case NW_ENOMEM: return "NW_ENOMEM: workspace allocation failed";
+    case NW_ECUDA: return "NW_ECUDA: a CUDA runtime call or workspace allocation failed (see nw_last_cuda_error)";
     case NW_ECOMM: return "NW_ECOMM: inconsistent sharded strip / halo description";
     default: return "NW_UNKNOWN";
   }

@@ -57,8 +57,11 @@ def test_library_is_sm100a_only():
 
 def test_status_strings(L):
     assert nwb.nw_status_str(NW_OK) == "NW_OK"
-    for s in range(1, 6):
+    for s in range(1, 5):
         assert nwb.nw_status_str(s).startswith("NW_E")
+    # NW_OK=0, NW_EINVAL=1, NW_ERANGE=2, NW_ECUDA=3, NW_ECOMM=4
+    assert (NW_OK, NW_EINVAL, NW_ERANGE, NW_ECUDA, NW_ECOMM) == (0, 1, 2, 3, 4)
+    assert nwb.nw_status_str(4).startswith("NW_ECOMM") and nwb.nw_status_str(5) == "NW_UNKNOWN"
     assert L.nw_abi_version() == 1
 
 
