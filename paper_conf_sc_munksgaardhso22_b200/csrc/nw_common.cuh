@@ -1,6 +1,6 @@
 // nw_common.cuh — definitions shared by the wavefront kernel (nw_wave.cuh) and the host side:
 // the band schedule (exported by nw_strip_map for pin P7), the kernel parameter block, the
-// border-source / sink kinds, small shared-memory / PTX helpers and the spin watchdog.
+// border-source / sink kinds, the volatile shared-memory accessors and the spin watchdog.
 //
 // What the path computes (Fig. 2, with Rodinia's cell function, R1):
 //     score[i][j] = max(score[i-1][j-1] + ref[i][j], score[i-1][j] - p, score[i][j-1] - p)
@@ -74,28 +74,10 @@ struct StripParams {
   int8_t subst[32 * 32];
 };
 
-__device__ __forceinline__ int prmt_sext(uint32_t w, uint32_t sel) {
-  uint32_t d;
-  asm("prmt.b32 %0, %1, 0, %2;" : "=r"(d) : "r"(w), "r"(sel));
-  return static_cast<int>(d);
-}
 // opaque copy: keeps a value in a register (stops the compiler re-deriving smem bases per step)
 __device__ __forceinline__ uint32_t opaque(uint32_t x) {
   asm volatile("mov.b32 %0, %0;" : "+r"(x));
   return x;
-}
-// ref-ring load: not volatile (the compiler may hoist it inside a staging block for ILP), but it
-// consumes the token produced after the chunk's mbarrier wait, so it never moves above it
-__device__ __forceinline__ int lds_tok(uint32_t a, uint32_t tok) {
-  int v;
-  asm("ld.shared.b32 %0, [%1];" : "=r"(v) : "r"(a), "r"(tok));
-  return v;
-}
-__device__ __forceinline__ uint32_t mbar_wait_tok(uint32_t bar, uint32_t parity) {
-  mbar_wait(bar, parity);
-  uint32_t tk;
-  asm volatile("mov.u32 %0, 0;" : "=r"(tk)::"memory");
-  return tk;
 }
 __device__ __forceinline__ uint64_t lds64_volatile(uint32_t a) {
   uint64_t v;
@@ -110,26 +92,6 @@ __device__ __forceinline__ int lds32_volatile(uint32_t a) {
 __device__ __forceinline__ void sts32_volatile(uint32_t a, int v) {
   asm volatile("st.volatile.shared.b32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
 }
-// predicated border-entry publishes (no branch in the step)
-__device__ __forceinline__ void st_entry_smem(bool pred, uint32_t a, uint32_t lo, uint32_t hi) {
-  asm volatile("{ .reg .pred q; .reg .b64 e; setp.ne.b32 q, %0, 0; mov.b64 e, {%2, %3}; @q st.volatile.shared.b64 [%1], e; }" ::"r"(
-                   static_cast<int>(pred)),
-               "r"(a), "r"(lo), "r"(hi)
-               : "memory");
-}
-__device__ __forceinline__ void st_entry_gpu(bool pred, uint64_t* p, uint32_t lo, uint32_t hi) {
-  asm volatile("{ .reg .pred q; .reg .b64 e; setp.ne.b32 q, %0, 0; mov.b64 e, {%2, %3}; @q st.relaxed.gpu.global.b64 [%1], e; }" ::"r"(
-                   static_cast<int>(pred)),
-               "l"(p), "r"(lo), "r"(hi)
-               : "memory");
-}
-__device__ __forceinline__ void st_entry_sys(bool pred, uint64_t* p, uint32_t lo, uint32_t hi) {
-  asm volatile("{ .reg .pred q; .reg .b64 e; setp.ne.b32 q, %0, 0; mov.b64 e, {%2, %3}; @q st.relaxed.sys.global.b64 [%1], e; }" ::"r"(
-                   static_cast<int>(pred)),
-               "l"(p), "r"(lo), "r"(hi)
-               : "memory");
-}
-
 __device__ __noinline__ void watchdog_trap(unsigned int* err) {
   atomicExch(err, kErrWatchdog);
   __trap();
@@ -138,8 +100,5 @@ __device__ __noinline__ void watchdog_trap(unsigned int* err) {
 // Border sources/sinks of one band (uniform per task)
 enum : int { kSrcPlain = 0, kSrcGlobal = 1, kSrcSmem = 2 };
 enum : int { kSinkNone = 0, kSinkSmem = 1, kSinkGlobal = 2 };
-
-// One band (task) of the persistent kernel; SINK is specialised so the steady-state step has no
-// branches.
 
 }  // namespace nwb200

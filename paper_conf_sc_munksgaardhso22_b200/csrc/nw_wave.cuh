@@ -112,10 +112,6 @@ struct WaveCfg {
 };
 
 // ---- inline PTX helpers (immediate offsets keep the per-step staging at one instruction per copy)
-template <int OFF>
-__device__ __forceinline__ void cp_async4_imm(uint32_t dst, uint64_t src) {
-  asm volatile("cp.async.ca.shared.global [%0+%2], [%1+%2], 4;" ::"r"(dst), "l"(src), "n"(OFF) : "memory");
-}
 template <int DOFF, int SOFF>
 __device__ __forceinline__ void cp_async4_imm2(uint32_t dst, uint64_t src) {
   asm volatile("cp.async.ca.shared.global [%0+%2], [%1+%3], 4;" ::"r"(dst), "l"(src), "n"(DOFF), "n"(SOFF) : "memory");
@@ -141,10 +137,6 @@ __device__ __forceinline__ int lds32_imm(uint32_t a) {
 template <int DBASE, int K>
 __device__ __forceinline__ void lds_row(uint32_t a0, int* v) {
   [&]<int... I>(std::integer_sequence<int, I...>) { ((v[I] = lds32_imm<DBASE + 128 * I>(a0)), ...); }(std::make_integer_sequence<int, K>{});
-}
-template <int OFF>
-__device__ __forceinline__ void sts32_imm(uint32_t a, int v) {
-  asm volatile("st.shared.b32 [%0+%2], %1;" ::"r"(a), "r"(v), "n"(OFF) : "memory");
 }
 template <int OFF>
 __device__ __forceinline__ void stg32_imm(uint64_t g, int v) {
