@@ -59,9 +59,6 @@ namespace nwb200 {
 #ifndef NW_PFC
 #define NW_PFC 12
 #endif
-#ifndef NW_SUB
-#define NW_SUB 8
-#endif
 #ifndef NW_PF_AT
 #define NW_PF_AT 8
 #endif
@@ -670,8 +667,23 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
 
   // one wavefront step s (entry jj of the block's border window); ALL = every lane's row is in
   // 1..n (no predicates)
+  constexpr int kPfAt = NW_PF_AT;  // mid-block work (border copy, progress pre-read) this many steps into the block
+  static_assert(kPfAt > 0 && kPfAt < CE, "mid-block point");
+  // the staging warps' progress words for the NEXT event, read kPfAt steps into the block
+  // (the result is first used at that event; cached values that already suffice are kept)
+  int cur_sig0 = 0;
+  auto pre_read = [&]() {
+    const int nl = SEQ ? 0 : min(n, cur_sig0 + 2 * CE + 1), ns = cur_sig0 + 2 * CE - SR;
+    if (landed < nl) {
+      int unused;
+      prog_read(from_r, landed, unused);
+    }
+    if (stored < ns) stored = read_stored();
+  };
   int vprev = 0;  // the out lane's previous row value (paired border-entry stores)
-  auto step = [&](const int s, const int jj, auto all_tag, auto par_tag) {
+  int vbuf[8];    // steady blocks: the out lane's last 8 row values, published as 4 pairs per 8 steps
+  auto step = [&](const int s, auto jj_tag, auto all_tag) {
+    constexpr int jj = decltype(jj_tag)::value;  // step within the block (an immediate)
     constexpr bool ALL = decltype(all_tag)::value;
     const int r = s + 1 - t;  // this lane's row
     // ---- ref of this step's row (loaded last step) and the next row's loads
@@ -694,6 +706,7 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     // ---- left value: lane t-1's last column of this row, lane 0: the border entry
     const int bval = __shfl_sync(FULL, curv, jj);
     const int from_left = __shfl_up_sync(FULL, vlast, 1);
+    if constexpr (jj == kPfAt) pre_read();  // (its acquire load waits in the shuffles' shadow)
     const int L = (t == 0) ? bval : from_left;
     bool active = true;
     if (!ALL) active = r >= 1 && r <= n;
@@ -724,10 +737,35 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
         for (int m = 0; m < K - 1; ++m) vo = out_m == m ? Pv[m] : vo;
       }
       if constexpr (HALO_OUT) vo -= out_adj + s * p;
-      if constexpr (!RAGGED && kPairs) {
+      if constexpr (!RAGGED && kPairs && ALL) {
+        // steady block (every row in 1..n, full band: the out lane is lane 31 at row r = s - 30):
+        // the out lane's values are buffered and published as four 16-byte pairs at the end of
+        // each 8-step half (rows r-7 .. r, r-7 even); one store per step held a register quad
+        // that the next step's store rewrote (ncu: long-scoreboard stalls behind the LSU queue)
+        vbuf[jj & 7] = vo;
+        if constexpr ((jj & 7) == 7) {
+#pragma unroll
+          for (int k = 0; k < 4; ++k) {
+            const int r0 = r - 7 + 2 * k;
+            const uint32_t u0 = static_cast<uint32_t>(r0);
+            if constexpr (REMOTE)
+              st_pair_dsmem_p(do_out && sink_smem, bring_out + 8u * (r0 & (C::BR - 1)), static_cast<uint32_t>(vbuf[2 * k]), gen | u0,
+                              static_cast<uint32_t>(vbuf[2 * k + 1]), gen | (u0 + 1));
+            else
+              st_pair_smem_p(do_out && sink_smem, bring_out + 8u * (r0 & (C::BR - 1)), static_cast<uint32_t>(vbuf[2 * k]), gen | u0,
+                             static_cast<uint32_t>(vbuf[2 * k + 1]), gen | (u0 + 1));
+            if constexpr (HALO_OUT)
+              st_pair_sys_p(do_out, lout + r0, static_cast<uint32_t>(vbuf[2 * k]), lout_tag, static_cast<uint32_t>(vbuf[2 * k + 1]), lout_tag);
+            else
+              st_pair_gpu_p(do_out && sink_gpu, lout + r0, static_cast<uint32_t>(vbuf[2 * k]), lout_tag, static_cast<uint32_t>(vbuf[2 * k + 1]),
+                            lout_tag);
+          }
+        }
+        vprev = vo;
+      } else if constexpr (!RAGGED && kPairs) {
         // full band: the out lane is lane 31, so its row r = s - 30 has the parity of J.  Odd
         // rows publish the pair (r-1, r) in one 16-byte store; an even last row is flushed alone.
-        constexpr bool ODD = decltype(par_tag)::value != 0;
+        constexpr bool ODD = (jj & 1) != 0;
         const uint32_t ur = static_cast<uint32_t>(r);
         if constexpr (ODD) {
           if constexpr (REMOTE)
@@ -768,13 +806,11 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     vlast = Pv[K - 1];
   };
 
-  constexpr int kSub = NW_SUB;    // steps per unrolled sub-block (a divisor of CE)
-  constexpr int kPfAt = NW_PF_AT;  // border copy issued this many steps into the block (a multiple of kSub)
-  static_assert(CE % kSub == 0 && kPfAt % kSub == 0 && kPfAt > 0 && kPfAt < CE, "sub-block geometry");
   const int nsteps = n + 31;  // compute steps 0 .. n+30
   const int nblk = (nsteps + CE - 1) / CE;
   for (int Q = 0; Q < nblk; ++Q) {
     const int sig0 = Q * CE;
+    cur_sig0 = sig0;
     // ---- event Q.  To the staging warp: ref rows <= sig0-30 consumed (lane 31 read row sig0-30
     // at step sig0-1), score rows <= sig0-31 complete (lane 31 wrote row sig0-31 at step sig0-1).
     const long long ce0 = tracing ? clock64() : 0;
@@ -865,41 +901,34 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
       const long long ce3 = clock64();
       ph_cyc[0] += ce1 - ce0, ph_cyc[1] += ce2 - ce1, ph_cyc[2] += ce3 - ce2;
     }
-    // ---- CE steps (two unrolled halves of CE/2)
+    // ---- CE steps, fully unrolled (the border entry index jj is an immediate), in two parts
+    // around the mid-block work at step kPfAt: the border copy of block Q + BD (global / plain
+    // sources) and a read of the staging warps' progress words for the NEXT event, whose result
+    // is consumed only there (its latency hides behind the second part's steps instead of
+    // stalling the event; measured ~200 cycles per event when read at the event itself)
+    auto mid_block = [&]() {
+      if constexpr (SRC != kSrcSmem) {
+        // a fresher snapshot of the producer's column than at the event (less band-to-band lag);
+        // later than the half point the L2 round trip is exposed at the event
+        if (sig0 + CE * BD < nsteps) prefetch_block(Q + BD);
+        cp_async_commit();
+      }
+    };
+    auto block_steps = [&](auto all_tag) {
+      [&]<int... J>(std::integer_sequence<int, J...>) {
+        (step(sig0 + J, std::integral_constant<int, J>{}, all_tag), ...);
+      }(std::make_integer_sequence<int, kPfAt>{});
+      mid_block();
+      [&]<int... J>(std::integer_sequence<int, J...>) {
+        (step(sig0 + kPfAt + J, std::integral_constant<int, kPfAt + J>{}, all_tag), ...);
+      }(std::make_integer_sequence<int, CE - kPfAt>{});
+    };
     if (sig0 >= 31 && sig0 + CE <= n) {
       const long long c0c = tracing ? clock64() : 0;
-#pragma unroll 1
-      for (int h = 0; h < CE; h += kSub) {
-        if constexpr (SRC != kSrcSmem) {
-          // the border copy of block Q + BD, issued kPfAt steps into the block before the event
-          // that first needs it (a fresher snapshot of the producer's column: less band-to-band
-          // lag; later than the half point the L2 round trip is exposed at the event)
-          if (h == kPfAt) {
-            if (sig0 + CE * BD < nsteps) prefetch_block(Q + BD);
-            cp_async_commit();
-          }
-        }
-        [&]<int... J>(std::integer_sequence<int, J...>) {
-          (step(sig0 + h + J, h + J, std::true_type{}, std::integral_constant<int, J & 1>{}), ...);
-        }(std::make_integer_sequence<int, kSub>{});
-      }
+      block_steps(std::true_type{});
       if (tracing) steady_cyc += clock64() - c0c, ++steady_blocks;
     } else {
-#pragma unroll 1
-      for (int h = 0; h < CE; h += kSub) {
-        if constexpr (SRC != kSrcSmem) {
-          // the border copy of block Q + BD, issued kPfAt steps into the block before the event
-          // that first needs it (a fresher snapshot of the producer's column: less band-to-band
-          // lag; later than the half point the L2 round trip is exposed at the event)
-          if (h == kPfAt) {
-            if (sig0 + CE * BD < nsteps) prefetch_block(Q + BD);
-            cp_async_commit();
-          }
-        }
-        [&]<int... J>(std::integer_sequence<int, J...>) {
-          (step(sig0 + h + J, h + J, std::false_type{}, std::integral_constant<int, J & 1>{}), ...);
-        }(std::make_integer_sequence<int, kSub>{});
-      }
+      block_steps(std::false_type{});
     }
   }
   prog_publish(to_s, n, n, !strict);  // every row consumed and complete
