@@ -50,6 +50,9 @@ struct StripParams {
   int64_t n;       // rows 1..n
   int64_t width;   // interior columns 1..width
   int32_t p;
+  int32_t vec16;  // 1: score and ref interior rows start 16-byte aligned (16-byte staging copies)
+  int32_t zero0;  // 0 (experiment builds: an operand the compiler cannot fold)
+  int32_t p2;  // 2p, read straight from the parameter bank by the step (a uniform operand, no register)
   int32_t nbands;  // bands per pair
   int64_t ntasks;  // pairs * nbands
   int64_t ngroups; // ceil(ntasks / NW) (pair mode: pairs)

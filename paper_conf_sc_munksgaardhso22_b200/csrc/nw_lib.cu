@@ -256,6 +256,7 @@ nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* 
   P.n = n;
   P.width = width;
   P.p = p;
+  P.p2 = 2 * p;
   P.nbands = static_cast<int32_t>(nbands);
   P.ntasks = pairs * nbands;
   const int var = tile_to_variant(tile);
@@ -274,6 +275,11 @@ nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* 
   }
   P.xbuf = w->xbuf;
   P.epoch = ++w->epoch;
+  // 16-byte staging copies when every interior row of score (and ref) starts 16-byte aligned
+  auto al16 = [&](const int32_t* base, int64_t ld, int64_t ps) {
+    return (reinterpret_cast<uintptr_t>(base + 1) & 15) == 0 && ld % 4 == 0 && (pairs == 1 || ps % 4 == 0);
+  };
+  P.vec16 = al16(score, lds, pss) && (SEQ || al16(ref, ldr, psr)) ? 1 : 0;
   P.halo_in = halo_in;
   P.halo_out = halo_out;
   P.halo_epoch = halo_epoch;

@@ -69,6 +69,11 @@ namespace nwb200 {
 #ifndef NW_DEBUG_SKIP
 #define NW_DEBUG_SKIP 0u
 #endif
+// NW_STEP_EXP (experiment builds only, results invalid): strip parts of the steady step to time
+// them -- 1 border-entry stores, 2 score-ring stores, 4 ref-ring loads, 8 border shuffle, 16 SEL
+#ifndef NW_STEP_EXP
+#define NW_STEP_EXP 0
+#endif
 #ifndef NW_STAGE_SLEEP_NS
 #define NW_STAGE_SLEEP_NS 0
 #endif
@@ -93,7 +98,11 @@ struct WaveCfg {
   static constexpr int PROF_WORDS = SEQ ? 32 * 32 * K : 0;  // int32 prof[x][lane][K] (+2p, gap-normalised)
   static constexpr int BPRE_BYTES = 4 * 8 * (CE + 2);  // border prefetch ring: 4 blocks x (CE+2) entries
   static constexpr int HDR_BYTES = 128;                // progress words: [0] compute -> staging, [8] ref -> compute, [16] store -> compute
-  static constexpr int NWARPS = NW * (1 + SPB);        // per band: a compute warp and SPB staging warps
+  // NW = 2, SPB = 2: eight warps so that the two compute warps (0, 1) have SM sub-partitions 0
+  // and 1 to themselves: ref warps 2, 3 and store warps 6, 7 share sub-partitions 2 and 3, warps
+  // 4 and 5 idle (with six warps the store warps 4, 5 took issue slots from the compute warps)
+  static constexpr bool SPREAD = NW == 2 && SPB == 2;
+  static constexpr int NWARPS = SPREAD ? 8 : NW * (1 + SPB);  // per band: a compute warp and SPB staging warps
   static constexpr size_t kWarpSmem = HDR_BYTES + 4ull * (REF_WORDS + SR * RS + PROF_WORDS) + BPRE_BYTES;
   // CTA header: ticket, progress words, the border rings between consecutive bands (NW - 1
   // between the warps of the CTA; CL > 1: one incoming ring written by the previous CTA)
@@ -124,6 +133,21 @@ __device__ __forceinline__ void cp_async4_imm_p(bool p, uint32_t dst, uint64_t s
                    static_cast<int>(p)),
                "r"(dst), "l"(src), "n"(OFF)
                : "memory");
+}
+// 16-byte forms for layouts whose interior rows start 16-byte aligned (StripParams::vec16)
+template <int DOFF, int SOFF>
+__device__ __forceinline__ void cp_async16_imm2(uint32_t dst, uint64_t src) {
+  asm volatile("cp.async.cg.shared.global [%0+%2], [%1+%3], 16;" ::"r"(dst), "l"(src), "n"(DOFF), "n"(SOFF) : "memory");
+}
+template <int OFF>
+__device__ __forceinline__ int4 lds128_imm(uint32_t a) {
+  int4 v;
+  asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4+%5];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a), "n"(OFF) : "memory");
+  return v;
+}
+template <int OFF>
+__device__ __forceinline__ void stg128_imm(uint64_t g, int4 v) {
+  asm volatile("st.global.v4.b32 [%0+%5], {%1, %2, %3, %4};" ::"l"(g), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w), "n"(OFF) : "memory");
 }
 template <int OFF>
 __device__ __forceinline__ int lds32_imm(uint32_t a) {
@@ -213,7 +237,7 @@ __device__ __forceinline__ void cluster_sync_all() {
   asm volatile("barrier.cluster.arrive.release.aligned; barrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
 
-enum : int { kRoleRef = 1, kRoleStore = 2 };  // staging-warp roles
+enum : int { kRoleRef = 1, kRoleStore = 2, kRoleIdle = 4 };  // staging-warp roles
 
 // Shared per-band geometry of the compute and staging warps.
 template <class C>
@@ -281,6 +305,7 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
   for (int i = 0; i < K; ++i) wmask |= static_cast<uint32_t>(32 * i + t < g.ws) << i;
   const uint64_t ldr4 = 4ull * static_cast<uint64_t>(P.ldr), lds4 = 4ull * static_cast<uint64_t>(P.lds);
   const uint64_t gR0 = SEQ ? 0ull : reinterpret_cast<uint64_t>(g.Rf + g.c0 + t);  // (row 0, word t) of the ref segment
+  const bool vec16 = P.vec16 != 0;  // interior rows 16-byte aligned: 16-byte copies / stores (host-checked)
   // progress words: release stores / acquire loads (NW_DEBUG_SKIP bit 4, experiment builds: relaxed;
   // measured: no difference, 3.08 vs 3.11 ms at n = 32768, 37.65 vs 37.53 ms on config 4)
   constexpr bool strict = (NW_DEBUG_SKIP & 16u) == 0;
@@ -296,7 +321,14 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
       const uint32_t d0 = g.refR + static_cast<uint32_t>((CH * k) & (RR - 1)) * RS4 + 4u * t;
       uint64_t gsrc = gR;
       gR += CH * ldr4;
-      if (!RAGGED && CH * k + CH <= n) {
+      if (!RAGGED && vec16 && CH * k + CH <= n) {
+        // 16-byte copies: lane t moves words 4t..4t+3 (+128: K = 8) of each row, 1 or 2 per row
+        const uint32_t dv = g.refR + static_cast<uint32_t>((CH * k) & (RR - 1)) * RS4 + 16u * t;
+        uint64_t gv = gsrc - 4ull * t + 16ull * t;
+        [&]<int... R>(std::integer_sequence<int, R...>) {
+          ((cp_async16_imm2<R * 4 * C::RS, 0>(dv, gv), (K == 8 ? cp_async16_imm2<R * 4 * C::RS + 512, 512>(dv, gv) : void()), gv += ldr4), ...);
+        }(std::make_integer_sequence<int, CH>{});
+      } else if (!RAGGED && CH * k + CH <= n) {
         [&]<int... R>(std::integer_sequence<int, R...>) {
           ((cp_row<R * 4 * C::RS, K>(d0, gsrc), gsrc += ldr4), ...);
         }(std::make_integer_sequence<int, CH>{});
@@ -342,13 +374,32 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
   int colp[K];
 #pragma unroll
   for (int I = 0; I < K; ++I) colp[I] = -(g.c0 + 32 * I + t) * g.p;
+  int cp16[K];  // 16-byte path: column terms of words 4t + j (+128)
+#pragma unroll
+  for (int j = 0; j < K; ++j) cp16[j] = -(g.c0 + 4 * t + (j & 3) + 128 * (j >> 2)) * g.p;
   uint64_t gS = gS0 + lds4 + (half > 0 ? CH * lds4 : 0ull);  // (row CH*ks+1, word t) of the next score chunk
   auto store_chunk = [&](int k) {
     const uint32_t a0 = g.scR + static_cast<uint32_t>((CH * k) & (SR - 1)) * RS4 + 4u * t;
     uint64_t ga = gS;
     gS += static_cast<uint64_t>(kstep * CH) * lds4;
     int rp = -(CH * k + 1) * g.p;
-    if (!RAGGED && CH * k + CH <= n) {
+    if (!RAGGED && vec16 && CH * k + CH <= n) {
+      // 16-byte path: LDS.128 of ring words 4t..4t+3 (+128), one IADD3 per value, STG.128
+      const uint32_t av = g.scR + static_cast<uint32_t>((CH * k) & (SR - 1)) * RS4 + 16u * t;
+      uint64_t gv = ga - 4ull * t + 16ull * t;
+#pragma unroll
+      for (int i = 0; i < CH; ++i) {
+        [&]<int... H>(std::integer_sequence<int, H...>) {
+          ((void)[&] {
+             int4 v = lds128_imm<H * 512>(av + static_cast<uint32_t>(i) * RS4);
+             v.x += rp + cp16[4 * H], v.y += rp + cp16[4 * H + 1], v.z += rp + cp16[4 * H + 2], v.w += rp + cp16[4 * H + 3];
+             stg128_imm<H * 512>(gv, v);
+           }(), ...);
+        }(std::make_integer_sequence<int, K / 4>{});
+        gv += lds4;
+        rp -= g.p;
+      }
+    } else if (!RAGGED && CH * k + CH <= n) {
       // the common case: K LDS + K IADD3 + K unpredicated coalesced STG per row
       int v[CH][K];
       [&]<int... R>(std::integer_sequence<int, R...>) { (lds_row<R * 4 * C::RS, K>(a0, v[R]), ...); }(std::make_integer_sequence<int, CH>{});
@@ -621,7 +672,6 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
   }
   const uint32_t profA = opaque(g.prof + 4u * K * t + 16u * sw);
 
-  const int p2 = 2 * p;
   uint32_t tok = 0;  // produced after each event's acquire, consumed by the ref loads
   int rvn[K];        // ref of the lane's NEXT row (loaded one step ahead)
 #pragma unroll
@@ -700,14 +750,14 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
       // ref' = ref + 2p (the diagonal move of the gap-normalised recurrence); off the
       // recurrence's critical path (the row was loaded one step ahead)
 #pragma unroll
-      for (int m = 0; m < K; ++m) rv[m] = rvn[m] + p2;
-      load_ref_row(laneR + static_cast<uint32_t>(r & (RR - 1)) * RS4);  // ring row of row r+1
+      for (int m = 0; m < K; ++m) rv[m] = rvn[m] + P.p2;
+      if constexpr (!(ALL && (NW_STEP_EXP & 4))) load_ref_row(laneR + static_cast<uint32_t>(r & (RR - 1)) * RS4);  // ring row of row r+1
     }
     // ---- left value: lane t-1's last column of this row, lane 0: the border entry
-    const int bval = __shfl_sync(FULL, curv, jj);
-    const int from_left = __shfl_up_sync(FULL, vlast, 1);
+    const int bval = (ALL && (NW_STEP_EXP & 8)) ? curv + jj : __shfl_sync(FULL, curv, jj);
+    const int from_left = (ALL && (NW_STEP_EXP & 128)) ? vlast + 1 : __shfl_up_sync(FULL, vlast, 1);
     if constexpr (jj == kPfAt) pre_read();  // (its acquire load waits in the shuffles' shadow)
-    const int L = (t == 0) ? bval : from_left;
+    const int L = (ALL && (NW_STEP_EXP & 16)) ? from_left + bval : (t == 0) ? bval : from_left;
     bool active = true;
     if (!ALL) active = r >= 1 && r <= n;
     if (active) {
@@ -715,6 +765,10 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
       // x_m = max(diag + ref', up); the row's left chain is a plain prefix max and the left
       // value L enters with one max per cell.
       int x[K];
+      if constexpr (ALL && (NW_STEP_EXP & 32)) {
+#pragma unroll
+        for (int m = 0; m < K; ++m) x[m] = 0;
+      }
       x[0] = __viaddmax_s32(Lprev, rv[0], Pv[0]);
 #pragma unroll
       for (int m = 1; m < K; ++m) x[m] = __viaddmax_s32(Pv[m - 1], rv[m], Pv[m]);
@@ -726,10 +780,17 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
       for (int m = 1; m < K; ++m) Y[m] = max(Y[m - 1], x[m]);
 #pragma unroll
       for (int m = 0; m < K; ++m) Pv[m] = max(L, Y[m]);
+      if constexpr (ALL && (NW_STEP_EXP & 32)) {  // (timing only) no recurrence chain: each cell independent
+#pragma unroll
+        for (int m = 0; m < K; ++m) Pv[m] = __viaddmax_s32(Pv[m], rv[m], L);
+      }
+      if constexpr (ALL && (NW_STEP_EXP & 64)) {  // (timing only) chain-free L path: S'_7 = max(L + 0, Y_7)
+        Pv[K - 1] = __viaddmax_s32(L, P.zero0, Y[K - 1]);
+      }
       Lprev = L;
       const uint32_t aS = laneS + static_cast<uint32_t>((r - 1) & (SR - 1)) * RS4;
       [&]<int... I>(std::integer_sequence<int, I...>) {
-        (sts128_ring<16 * I>(aS, Pv[4 * I], Pv[4 * I + 1], Pv[4 * I + 2], Pv[4 * I + 3]), ...);
+        if constexpr (!(ALL && (NW_STEP_EXP & 2))) (sts128_ring<16 * I>(aS, Pv[4 * I], Pv[4 * I + 1], Pv[4 * I + 2], Pv[4 * I + 3]), ...);
       }(std::make_integer_sequence<int, K / 4>{});
       int vo = Pv[K - 1];
       if constexpr (RAGGED) {
@@ -737,7 +798,8 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
         for (int m = 0; m < K - 1; ++m) vo = out_m == m ? Pv[m] : vo;
       }
       if constexpr (HALO_OUT) vo -= out_adj + s * p;
-      if constexpr (!RAGGED && kPairs && ALL) {
+      if constexpr (ALL && (NW_STEP_EXP & 1)) {
+      } else if constexpr (!RAGGED && kPairs && ALL) {
         // steady block (every row in 1..n, full band: the out lane is lane 31 at row r = s - 30):
         // the out lane's values are buffered and published as four 16-byte pairs at the end of
         // each 8-step half (rows r-7 .. r, r-7 even); one store per step held a register quad
@@ -960,8 +1022,9 @@ __global__ void __launch_bounds__(32 * C::NWARPS, 1) nw_wave_kernel(const __grid
   // 2NW..3NW-1 store staging
   const int wa = threadIdx.x >> 5;
   const bool staging = wa >= NW;
-  const int role = wa < NW ? 0 : (C::SPB == 1 ? (kRoleRef | kRoleStore) : (wa < 2 * NW ? kRoleRef : kRoleStore));
+  int role = wa < NW ? 0 : (C::SPB == 1 ? (kRoleRef | kRoleStore) : (wa < 2 * NW ? kRoleRef : kRoleStore));
   const int half = C::SPB == 3 && wa >= 2 * NW ? (wa >= 3 * NW ? 1 : 0) : -1;  // SPB = 3: even / odd score chunks
+  if (C::SPREAD && wa >= 2 * NW) role = wa >= 6 ? kRoleStore : kRoleIdle;
   const int w = wa % NW;  // the band slot this warp serves
   // CTA header: [0] group ticket, [8 + 4w] consumer progress of warp w, [128..] border rings
   unsigned long long* const s_group = reinterpret_cast<unsigned long long*>(smem);
@@ -1007,7 +1070,8 @@ __global__ void __launch_bounds__(32 * C::NWARPS, 1) nw_wave_kernel(const __grid
     if (task < P.ntasks) {
       const int band = static_cast<int>(task % P.nbands);
       const bool full = band_ws(P.width, band, C::W) == C::W;
-      if (C::SPB == 1 && staging) {
+      if (role == kRoleIdle) {
+      } else if (C::SPB == 1 && staging) {
         if (full)
           wave_stage<C, false, kRoleRef | kRoleStore>(P, task, t, wsm);
         else

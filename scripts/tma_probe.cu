@@ -16,7 +16,9 @@ constexpr int ROWS = 64;
 #endif
 constexpr int BOX = BOXW;
 
-__global__ void k(const __grid_constant__ CUtensorMap tm, int stride_b, int c0, int ld, int* bad, long long* cyc) {
+// MODE 0: tensor map as a __grid_constant__ parameter; 1: tensor map in global memory (tmg);
+// 2: plain 1-D bulk copy (cp.async.bulk, 16-byte aligned source: c0 rounded down)
+__global__ void k(const __grid_constant__ CUtensorMap tm, const CUtensorMap* tmg, int mode, int stride_b, int c0, int ld, int* bad, long long* cyc, const int* gsrc) {
   extern __shared__ __align__(1024) unsigned char sm[];
   __shared__ __align__(8) unsigned long long bar;
   const unsigned b = static_cast<unsigned>(__cvta_generic_to_shared(&bar));
@@ -31,10 +33,16 @@ __global__ void k(const __grid_constant__ CUtensorMap tm, int stride_b, int c0, 
     for (int r = 0; r < ROWS; ++r) {
       const unsigned dst = static_cast<unsigned>(__cvta_generic_to_shared(sm + r * stride_b));
       const int x = (r & 3) * ld + c0, y = r >> 2;
-      asm volatile(
-          "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(dst),
-          "l"(reinterpret_cast<unsigned long long>(&tm)), "r"(x), "r"(y), "r"(b)
-          : "memory");
+      if (mode == 2) {
+        const int* src = gsrc + (static_cast<long long>(r) * ld + c0) / 4 * 4;
+        asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst), "l"(src), "r"(BOX * 4), "r"(b) : "memory");
+      } else {
+        const unsigned long long tmap = mode == 0 ? reinterpret_cast<unsigned long long>(&tm) : reinterpret_cast<unsigned long long>(tmg);
+        asm volatile(
+            "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(dst),
+            "l"(tmap), "r"(x), "r"(y), "r"(b)
+            : "memory");
+      }
     }
   }
   long long t1 = clock64();
@@ -48,7 +56,8 @@ __global__ void k(const __grid_constant__ CUtensorMap tm, int stride_b, int c0, 
   for (int r = 0; r < ROWS; ++r)
     for (int c = threadIdx.x; c < BOX; c += blockDim.x) {
       const int v = reinterpret_cast<const int*>(sm + r * stride_b)[c];
-      const int want = (c0 + c < ld) ? r * 100000 + c0 + c : -1;  // beyond the row: ignore
+      const int cc = mode == 2 ? (r * ld + c0) / 4 * 4 - r * ld + c : c0 + c;  // (bulk: aligned-down start)
+      const int want = (cc >= 0 && cc < ld) ? r * 100000 + cc : -1;  // beyond the row: ignore
       if (want >= 0 && v != want) ++nb;
     }
   atomicAdd(bad, nb);
@@ -58,6 +67,7 @@ __global__ void k(const __grid_constant__ CUtensorMap tm, int stride_b, int c0, 
 int main(int argc, char** argv) {
   const int stride_b = argc > 1 ? atoi(argv[1]) : 1024;
   const int c0 = argc > 2 ? atoi(argv[2]) : 1;
+  const int mode = argc > 3 ? atoi(argv[3]) : 0;
   const int n = 1024, ld = n + 1;  // odd pitch: rows start at every 4-byte phase
   int* h = (int*)malloc(sizeof(int) * (n + 1) * ld);
   for (int r = 0; r <= n; ++r)
@@ -83,13 +93,16 @@ int main(int argc, char** argv) {
   if (cr != CUDA_SUCCESS) { printf("encode failed %d\n", (int)cr); return 1; }
   const int smem = ROWS * stride_b + 1024;
   cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  k<<<1, 128, smem>>>(tm, stride_b, c0, ld, bad, cyc);
+  CUtensorMap* tmg = nullptr;
+  cudaMalloc(&tmg, sizeof(CUtensorMap));
+  cudaMemcpy(tmg, &tm, sizeof(CUtensorMap), cudaMemcpyHostToDevice);
+  k<<<1, 128, smem>>>(tm, tmg, mode, stride_b, c0, ld, bad, cyc, d);
   cudaError_t e = cudaDeviceSynchronize();
   int hb = -1;
   long long hc[2] = {0, 0};
   cudaMemcpy(&hb, bad, 4, cudaMemcpyDeviceToHost);
   cudaMemcpy(hc, cyc, 16, cudaMemcpyDeviceToHost);
-  printf("stride %d B, c0 %d: %s, mismatches %d, issue %lld cyc for %d TMA, landed after %lld cyc\n", stride_b, c0,
+  printf("mode %d stride %d B, c0 %d: %s, mismatches %d, issue %lld cyc for %d TMA, landed after %lld cyc\n", mode, stride_b, c0,
          e == cudaSuccess ? "ok" : cudaGetErrorString(e), hb, hc[0], ROWS, hc[1]);
   return 0;
 }

@@ -18,10 +18,19 @@ __device__ __forceinline__ int imad(int a, int b, int c) {
   return d;
 }
 
-template <int F>
-__global__ void __launch_bounds__(32, 1) k(int* out, long long* cyc, const __grid_constant__ Prm P) {
+template <int F, int POLL = 0>
+__global__ void __launch_bounds__(128, 1) k(int* out, long long* cyc, const __grid_constant__ Prm P) {
   extern __shared__ __align__(16) int sm[];
   const int t = threadIdx.x & 31;
+  if (threadIdx.x >= 32) {  // POLL warps: spin on a shared word until the compute warp is done
+    if (threadIdx.x / 32 > POLL) return;
+    volatile int* flag = sm + 2 * RR * RS + 64;
+    int acc = 0;
+    while (flag[0] == 0) acc += flag[1];
+    if (acc == 12345) out[0] = acc;
+    return;
+  }
+  if (t == 0) sm[2 * RR * RS + 64] = 0;
   for (int i = t; i < 2 * RR * RS + 64; i += 32) sm[i] = (i * 7) % 13 - 4;
   __syncwarp();
   const unsigned base = static_cast<unsigned>(__cvta_generic_to_shared(sm + 64));
@@ -52,7 +61,7 @@ __global__ void __launch_bounds__(32, 1) k(int* out, long long* cyc, const __gri
       if constexpr (F == 7) {  // no SHFL.IDX
         bval = curv + jj;
         fl = __shfl_up_sync(0xffffffffu, vlast, 1);
-      } else if constexpr (F == 8) {  // no shuffle at all
+      } else if constexpr (F == 8 || F == 15 || F == 16) {  // no shuffle at all
         bval = curv + jj;
         fl = vlast + 1;
       } else if constexpr (F == 9) {  // two SHFL.UP, no SHFL.IDX
@@ -132,6 +141,39 @@ __global__ void __launch_bounds__(32, 1) k(int* out, long long* cyc, const __gri
           D = up;
           Pv[m] = __float_as_int(fmaxf(__int_as_float(L) + __int_as_float(z[m]), Y));
         }
+      } else if constexpr (F == 13 || F == 15) {  // tree prefix (z on level-2/3 nodes), x = VIADDMNMX(diag, ref+p2, up), S = max(L, Y)
+        int x[K], Y[K];
+        const int p2 = P.p2;
+        x[0] = __viaddmax_s32(Lprev, rv[0] + p2, Pv[0]);
+#pragma unroll
+        for (int m = 1; m < K; ++m) x[m] = __viaddmax_s32(Pv[m - 1], rv[m] + p2, Pv[m]);
+        const int m01 = max(x[0], x[1]), m23 = max(x[2], x[3]), m45 = max(x[4], x[5]), m67 = max(x[6], x[7]);
+        Y[0] = x[0];
+        Y[1] = m01;
+        Y[2] = __viaddmax_s32(m01, z[0], x[2]);
+        Y[3] = __viaddmax_s32(m01, z[1], m23);
+        const int m46 = __viaddmax_s32(m45, z[2], x[6]), m47 = __viaddmax_s32(m45, z[3], m67);
+        Y[4] = __viaddmax_s32(Y[3], z[4], x[4]);
+        Y[5] = __viaddmax_s32(Y[3], z[5], m45);
+        Y[6] = __viaddmax_s32(Y[3], z[6], m46);
+        Y[7] = __viaddmax_s32(Y[3], z[7], m47);
+        const int LL = F == 15 ? fl : L;
+#pragma unroll
+        for (int m = 0; m < K; ++m) Pv[m] = max(LL, Y[m]);
+      } else if constexpr (F == 14 || F == 16) {  // two half chains + combine
+        int x[K], Y[K];
+        const int p2 = P.p2;
+        x[0] = __viaddmax_s32(Lprev, rv[0] + p2, Pv[0]);
+#pragma unroll
+        for (int m = 1; m < K; ++m) x[m] = __viaddmax_s32(Pv[m - 1], rv[m] + p2, Pv[m]);
+        Y[0] = x[0];
+        for (int m = 1; m < 4; ++m) Y[m] = max(Y[m - 1], x[m]);
+        int Z = x[4];
+        Y[4] = __viaddmax_s32(Y[3], z[4], Z);
+        for (int m = 5; m < 8; ++m) { Z = max(Z, x[m]); Y[m] = __viaddmax_s32(Y[3], z[m], Z); }
+        const int LL = F == 16 ? fl : L;
+#pragma unroll
+        for (int m = 0; m < K; ++m) Pv[m] = max(LL, Y[m]);
       } else if constexpr (F == 4) {  // raw ref: x = max(IADD3(diag, ref, 2p), up), S chained
         int S = L, D = Lprev;
 #pragma unroll
@@ -173,6 +215,7 @@ __global__ void __launch_bounds__(32, 1) k(int* out, long long* cyc, const __gri
     }
   }
   long long t1 = clock64();
+  if (t == 0) sm[2 * RR * RS + 64] = 1;
   int acc = 0;
 #pragma unroll
   for (int m = 0; m < K; ++m) acc ^= Pv[m];
@@ -180,20 +223,20 @@ __global__ void __launch_bounds__(32, 1) k(int* out, long long* cyc, const __gri
   if (t == 0) cyc[blockIdx.x] = t1 - t0;
 }
 
-template <int F>
+template <int F, int POLL = 0>
 void run(const char* name, int* out, long long* cyc) {
   Prm P{};
   P.one = 1;
   P.p2 = 20;
   for (int i = 0; i < 8; ++i) P.z[i] = 0;
-  const int smem = 4 * (2 * RR * RS + 64);
-  cudaFuncSetAttribute(k<F>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  k<F><<<148, 32, smem>>>(out, cyc, P);
-  k<F><<<148, 32, smem>>>(out, cyc, P);
+  const int smem = 4 * (2 * RR * RS + 64 + 4);
+  cudaFuncSetAttribute(k<F, POLL>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  k<F, POLL><<<148, 32 * (1 + POLL), smem>>>(out, cyc, P);
+  k<F, POLL><<<148, 32 * (1 + POLL), smem>>>(out, cyc, P);
   cudaError_t e = cudaDeviceSynchronize();
   long long h = 0;
   cudaMemcpy(&h, cyc, 8, cudaMemcpyDeviceToHost);
-  printf("F=%d %-62s %6.1f cyc/step %s\n", F, name, static_cast<double>(h) / NSTEP, e == cudaSuccess ? "" : cudaGetErrorString(e));
+  printf("F=%d P=%d %-60s %6.1f cyc/step %s\n", F, POLL, name, static_cast<double>(h) / NSTEP, e == cudaSuccess ? "" : cudaGetErrorString(e));
 }
 
 int main() {
@@ -214,5 +257,12 @@ int main() {
   run<10>("fp32: FADD d, FMNMX3 Y chain, FMNMX(L+z, Y)", out, cyc);
   run<11>("fp32 chained: S = FMNMX3(S, d, up)", out, cyc);
   run<12>("fp32: 2-input FMNMX Y, FMNMX(L+z, Y)", out, cyc);
+  run<13>("tree prefix (z on L2/L3 nodes), S = max(L, Y)", out, cyc);
+  run<14>("two half chains + combine, S = max(L, Y)", out, cyc);
+  run<15>("tree prefix, no shuffles", out, cyc);
+  run<16>("two half chains, no shuffles", out, cyc);
+  run<1, 1>("round-1 form + 1 warp polling a shared word", out, cyc);
+  run<1, 3>("round-1 form + 3 warps polling a shared word", out, cyc);
+  run<8, 3>("no shuffles + 3 polling warps", out, cyc);
   return 0;
 }
