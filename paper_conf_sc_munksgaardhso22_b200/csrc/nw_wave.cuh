@@ -533,7 +533,12 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
   constexpr uint32_t RS4 = 4u * C::RS;
   constexpr bool SEQ = C::SEQ;
   constexpr unsigned FULL = 0xffffffffu;
-  constexpr int BD = SRC == kSrcGlobal ? 1 : 3;  // border prefetch distance (blocks)
+  // border prefetch distance (blocks): a polled global source (the previous band still running)
+  // is copied one block ahead -- an older snapshot would add its age to the band-to-band lag; a
+  // complete source (the input column, or in pair mode the finished previous band, whose entries
+  // come back from HBM) three blocks ahead so the copy's latency is hidden (one block ahead exposed
+  // ~350 cycles per event on config 4)
+  const int BD = (SRC == kSrcGlobal && !P.pair_mode) ? 1 : 3;
   const bool tracing = kTrace && P.trace != nullptr;
   const unsigned long long t_task0 = tracing ? globaltimer_ns() : 0ull;
   long long spin_cyc = 0, wait_cyc = 0, bp_cyc = 0, steady_cyc = 0, steady_blocks = 0;
