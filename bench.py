@@ -228,6 +228,8 @@ def main():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--layout", default="rodinia", choices=["rodinia", "aligned"],
                     help="matrix layout: pitch n+1 (Rodinia) or 16-byte aligned interior rows")
+    ap.add_argument("--cluster", action="store_true",
+                    help="experiment: one pair as thread-block clusters handing the border over through DSMEM")
     ap.add_argument("--trace", default="", help="write per-band {task,start,end,smid} of one extra launch here (.npy)")
     ap.add_argument("--variant", default="strip", choices=["strip", "diagonal", "unopt", "seq"],
                     help="ablation: the paper's per-diagonal structure (Opt) / Unopt instead of the "
@@ -251,6 +253,8 @@ def main():
     import paper_conf_sc_munksgaardhso22_b200 as nwb
     torch.cuda.set_device(local_rank)
     dev = torch.device("cuda", local_rank)
+    if args.cluster:
+        nwb.nw_debug_set_cluster(True)
     if world > 1:
         import torch.distributed as dist
         dist.init_process_group("nccl", device_id=dev)

@@ -60,7 +60,7 @@ namespace nwb200 {
 #define NW_PFC 12
 #endif
 #ifndef NW_PF_AT
-#define NW_PF_AT 8
+#define NW_PF_AT 4
 #endif
 // Experiment builds only (scripts/, _build.build_variant): NW_DEBUG_SKIP skips parts of the
 // staging (bits 0-3: results invalid), relaxes the progress words (bit 4) or switches the L2
