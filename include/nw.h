@@ -33,8 +33,12 @@
  *     b in {16, 32, 64, 128} -> W = 128 (K = 4; narrower b x b tiles are processed 128/b side
  *     by side, because a lane's K ref values are 16-byte shared loads).  A CTA owns one band
  *     (b in {0, 256, 32, 64}: a compute warp, a ref-staging warp and two store warps) or two
- *     consecutive bands (b in {16, 128}: two compute warps, a ref and a store warp each).
- *     The result does not depend on it (R8).
+ *     consecutive bands (b in {16, 128}: two compute warps on SM sub-partitions of their own,
+ *     a ref and a store warp each on the other two).  The result does not depend on it
+ *     (R8).
+ *   - Layouts whose interior rows start 16-byte aligned ((base + 1) % 16 == 0, ld % 4 == 0,
+ *     pair strides % 4 == 0, for score and ref) are staged with 16-byte copies and stores; any
+ *     other 4-byte aligned layout (e.g. the Rodinia pitch n + 1) with 4-byte copies.  Same result.
  *   - Any n >= 0 is accepted (ragged last band: n need not be a multiple of b).
  *   - Validation is synchronous and happens before anything is enqueued.  Range contract:
  *     0 <= penalty and (n+1)*(2*penalty + NW_REF_MAX) < 2^30 (else NW_ERANGE); |ref| <= NW_REF_MAX

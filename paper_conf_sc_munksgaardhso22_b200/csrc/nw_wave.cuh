@@ -59,6 +59,9 @@ namespace nwb200 {
 #ifndef NW_PFC
 #define NW_PFC 12
 #endif
+#ifndef NW_BD_GLOBAL
+#define NW_BD_GLOBAL 1  // border prefetch distance (blocks) of a polled global source
+#endif
 #ifndef NW_PF_AT
 #define NW_PF_AT 4
 #endif
@@ -538,7 +541,7 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
   // complete source (the input column, or in pair mode the finished previous band, whose entries
   // come back from HBM) three blocks ahead so the copy's latency is hidden (one block ahead exposed
   // ~350 cycles per event on config 4)
-  const int BD = (SRC == kSrcGlobal && !P.pair_mode) ? 1 : 3;
+  const int BD = (SRC == kSrcGlobal && !P.pair_mode) ? NW_BD_GLOBAL : 3;
   const bool tracing = kTrace && P.trace != nullptr;
   const unsigned long long t_task0 = tracing ? globaltimer_ns() : 0ull;
   long long spin_cyc = 0, wait_cyc = 0, bp_cyc = 0, steady_cyc = 0, steady_blocks = 0;
