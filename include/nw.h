@@ -150,11 +150,13 @@ nw_status nw_fill_seq_batch(int32_t* score, int64_t ld_score, int64_t stride_sco
 
 /* ---- end to end from HOST memory (bench e2e) ---------------------------------------
  * Copies ref (rows 1..n) and the borders host->device, runs nw_fill, copies the full score
- * matrix device->host.  Host buffers: (n+1)x(n+1) int32, pitch n+1.  Pinned (device-mapped)
- * buffers take the zero-copy path: the kernel reads ref and writes score over the host link
- * directly, both directions overlapped with the wavefront (NW_HOST_ZEROCOPY=0 disables);
- * pageable buffers are staged through cached device buffers.  Synchronous: returns when
- * score_host holds the result.  Device buffers are freed by nw_release_workspace(). */
+ * matrix device->host.  Host buffers: (n+1)x(n+1) int32, pitch n+1.  Pinned buffers take a
+ * copy-engine pipeline: ref moves host->device in ~32 MB row blocks on one stream while the
+ * kernel runs (its ref warps wait for the blocks they stage), and each score row block moves
+ * back on a second stream as soon as every band has stored it (stream memory operations on
+ * device counters), so both link directions and the wavefront overlap.  Pageable buffers are
+ * staged (copy in, fill, copy out).  Synchronous: returns when score_host holds the result.
+ * Device buffers are freed by nw_release_workspace(). */
 nw_status nw_fill_host(int32_t* score_host, const int32_t* ref_host, int64_t n, int32_t penalty,
                        int32_t tile, int32_t device);
 /* nw_fill_batch_host: the same for `batch` independent pairs stored back to back
@@ -229,10 +231,15 @@ void nw_debug_set_grid(int32_t grid);
  *     -1 = never;
  *   nw_debug_set_cluster(on): single pairs on the K = 8 kernel as thread-block clusters handing the
  *     border column over through distributed shared memory (measured slower; off by default);
- *   nw_debug_set_host_zero_copy(on): nw_fill[_batch]_host runs the kernel directly on pinned host
- *     buffers (default 1) instead of staging them in device memory. */
+ *   nw_debug_set_host_mode(mode): how nw_fill[_batch]_host treats PINNED host buffers: 2 = the
+ *     copy-engine pipeline (default), 1 = zero copy (the kernel reads ref and writes score over the
+ *     host link itself), 0 = staged (copy in, fill, copy out);
+ *   nw_debug_set_host_block_rows(rows): the pipeline's row-block size (0 = automatic, ~64 MB);
+ *   nw_debug_set_host_zero_copy(on): shorthand for nw_debug_set_host_mode(on ? 1 : 2). */
 void nw_debug_set_pair_mode(int32_t mode);
 void nw_debug_set_cluster(int32_t on);
+void nw_debug_set_host_mode(int32_t mode);
+void nw_debug_set_host_block_rows(int64_t rows);
 void nw_debug_set_host_zero_copy(int32_t on);
 
 /* Debug hook: persistent-kernel launches record, per task (pair, band) t < cap_tasks, eight

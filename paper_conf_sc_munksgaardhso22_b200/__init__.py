@@ -24,7 +24,8 @@ __all__ = [
     "NwError", "lib", "nw_fill", "nw_fill_batch", "nw_fill_seq", "nw_fill_seq_batch", "nw_fill_sharded", "nw_fill_host", "nw_fill_batch_host",
     "nw_fill_diagonal", "nw_fill_unopt", "nw_traceback", "nw_traceback_batch", "nw_band_width", "nw_launch_count", "nw_diag_lmad",
     "nw_kernel_info", "nw_strip_map", "nw_debug_set_grid", "nw_debug_set_trace", "nw_release_workspace", "nw_status_str",
-    "nw_debug_set_pair_mode", "nw_debug_set_cluster", "nw_debug_set_host_zero_copy",
+    "nw_debug_set_pair_mode", "nw_debug_set_cluster", "nw_debug_set_host_zero_copy", "nw_debug_set_host_mode",
+    "nw_debug_set_host_block_rows",
 ]
 
 NW_OK, NW_EINVAL, NW_ERANGE, NW_ECUDA, NW_ECOMM = range(5)  # SURVEY.md §8(b) numbering
@@ -96,9 +97,11 @@ def lib() -> ctypes.CDLL:
             L.nw_debug_set_trace.restype = None
             L.nw_debug_set_grid.argtypes = [_i32]
             L.nw_debug_set_grid.restype = None
-            for f in ("nw_debug_set_pair_mode", "nw_debug_set_cluster", "nw_debug_set_host_zero_copy"):
+            for f in ("nw_debug_set_pair_mode", "nw_debug_set_cluster", "nw_debug_set_host_zero_copy", "nw_debug_set_host_mode"):
                 getattr(L, f).argtypes = [_i32]
                 getattr(L, f).restype = None
+            L.nw_debug_set_host_block_rows.argtypes = [_i64]
+            L.nw_debug_set_host_block_rows.restype = None
             L.nw_release_workspace.restype = None
             for f in ("nw_fill", "nw_fill_ld", "nw_fill_batch", "nw_fill_batch_ld", "nw_fill_sharded",
                       "nw_fill_host", "nw_fill_batch_host", "nw_fill_diagonal", "nw_fill_unopt", "nw_kernel_info", "nw_fill_seq",
@@ -363,6 +366,16 @@ def nw_debug_set_cluster(on: bool):
 
 def nw_debug_set_host_zero_copy(on: bool):
     lib().nw_debug_set_host_zero_copy(int(bool(on)))
+
+
+def nw_debug_set_host_block_rows(rows: int):
+    """Row-block size of the host pipeline (0: automatic, ~64 MB)."""
+    lib().nw_debug_set_host_block_rows(int(rows))
+
+
+def nw_debug_set_host_mode(mode: int):
+    """Pinned host buffers in nw_fill[_batch]_host: 2 copy-engine pipeline (default), 1 zero copy, 0 staged."""
+    lib().nw_debug_set_host_mode(int(mode))
 
 
 def nw_debug_set_trace(buf=None):

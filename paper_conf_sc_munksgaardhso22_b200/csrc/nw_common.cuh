@@ -50,6 +50,12 @@ struct StripParams {
   int64_t n;       // rows 1..n
   int64_t width;   // interior columns 1..width
   int32_t p;
+  // host pipeline (nw_fill[_batch]_host, pinned buffers): the stacked matrix's rows (pair * (n+1)
+  // + r) in blocks of chunk_rows; ref block arrivals counted in *ref_ready by the copy-in stream,
+  // score block completions counted per block in rows_done by the store warps (null: off)
+  const unsigned* ref_ready;
+  unsigned* rows_done;
+  int64_t chunk_rows;
   int32_t vec16;  // 1: score and ref interior rows start 16-byte aligned (16-byte staging copies)
   int32_t zero0;  // 0 (experiment builds: an operand the compiler cannot fold)
   int32_t p2;  // 2p, read straight from the parameter bank by the step (a uniform operand, no register)

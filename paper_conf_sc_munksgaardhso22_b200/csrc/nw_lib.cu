@@ -4,6 +4,7 @@
 // band-border buffer, Unopt temporary), and the launches.  Every compute step runs in the
 // kernels of nw_wave.cuh / nw_diag.cuh; there is no CPU fallback: without a usable CUDA
 // device the entry points return NW_ECUDA.
+#include <cuda.h>
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -126,7 +127,8 @@ DevInfo g_dev[128];
 int g_debug_grid = 0;
 bool g_debug_cluster = false;
 int g_debug_pair_mode = 0;
-bool g_host_zero_copy = true;
+int g_host_mode = 2;  // pinned host buffers: 0 staged, 1 zero copy, 2 copy-engine pipeline
+int64_t g_host_block_rows = 0;  // pipeline row-block size (0: ~64 MB)
 unsigned long long* g_trace = nullptr;
 long long g_trace_cap = 0;
 
@@ -222,12 +224,19 @@ unsigned long long spin_limit_ns() {
   return v;
 }
 
+// Host pipeline signals (nw_fill[_batch]_host on pinned buffers, see there)
+struct HostPipe {
+  const unsigned* ref_ready;
+  unsigned* rows_done;
+  int64_t chunk_rows;
+};
+
 // One launch of the persistent kernel over `pairs` x ceil(width/W) bands.
 nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* ref, int64_t ldr, int64_t psr,
                        int64_t pairs, int64_t n, int64_t width, int32_t p, int32_t tile, const uint64_t* halo_in,
                        uint64_t* halo_out, uint32_t halo_epoch, int32_t halo_out_sys, cudaStream_t st,
                        const uint8_t* seq_a = nullptr, const uint8_t* seq_b = nullptr, int64_t psa = 0,
-                       int64_t psb = 0, const int8_t* subst32 = nullptr) {
+                       int64_t psb = 0, const int8_t* subst32 = nullptr, const HostPipe* pipe = nullptr) {
   const int K = tile_to_k(tile);
   const bool SEQ = seq_a != nullptr;
   const int W = 32 * K;
@@ -280,6 +289,11 @@ nw_status launch_strip(int32_t* score, int64_t lds, int64_t pss, const int32_t* 
     return (reinterpret_cast<uintptr_t>(base + 1) & 15) == 0 && ld % 4 == 0 && (pairs == 1 || ps % 4 == 0);
   };
   P.vec16 = al16(score, lds, pss) && (SEQ || al16(ref, ldr, psr)) ? 1 : 0;
+  if (pipe) {
+    P.ref_ready = pipe->ref_ready;
+    P.rows_done = pipe->rows_done;
+    P.chunk_rows = pipe->chunk_rows;
+  }
   P.halo_in = halo_in;
   P.halo_out = halo_out;
   P.halo_epoch = halo_epoch;
@@ -402,7 +416,27 @@ struct HostBufs {
   int32_t* ref = nullptr;
   size_t elems = 0;
   cudaStream_t st = nullptr;
+  cudaStream_t sin = nullptr, sout = nullptr;  // pipeline: copy-in / copy-out streams
+  cudaEvent_t ev = nullptr;
+  unsigned* flags = nullptr;  // pipeline: [0] ref blocks arrived, [1 + c] store signals of block c
+  size_t nflags = 0;
 };
+
+// Stream memory operations (driver API, fetched at run time: the library links only cudart)
+using PfnWaitValue32 = CUresult (*)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+using PfnWriteValue32 = CUresult (*)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+PfnWaitValue32 g_wait_value = nullptr;
+PfnWriteValue32 g_write_value = nullptr;
+bool stream_mem_ops() {
+  static const bool ok = [] {
+    cudaDriverEntryPointQueryResult q;
+    cudaGetDriverEntryPoint("cuStreamWaitValue32", reinterpret_cast<void**>(&g_wait_value), cudaEnableDefault, &q);
+    cudaGetDriverEntryPoint("cuStreamWriteValue32", reinterpret_cast<void**>(&g_write_value), cudaEnableDefault, &q);
+    (void)cudaGetLastError();
+    return g_wait_value != nullptr && g_write_value != nullptr;
+  }();
+  return ok;
+}
 HostBufs g_host[128];
 // one staged host call per device at a time: the staging buffers and their stream are per device
 // (the lock spans the reallocation, the copies, the launch and the final synchronisation)
@@ -520,24 +554,22 @@ nw_status nw_fill_batch_host(int32_t* score_host, const int32_t* ref_host, int64
     std::lock_guard<std::mutex> lk(g_mu);
     if (!hb.st) NW_CU(cudaStreamCreateWithFlags(&hb.st, cudaStreamNonBlocking));
   }
-  // Pinned (device-mapped) host buffers: the kernel streams ref in and score out over the host
-  // link itself (zero copy, both directions at once, overlapped with the wavefront) instead of
-  // copy-in / compute / copy-out.  Pageable buffers take the staged path below.
-  if (g_host_zero_copy) {
-    cudaPointerAttributes as{}, ar{};
-    const bool ok = cudaPointerGetAttributes(&as, score_host) == cudaSuccess &&
-                    cudaPointerGetAttributes(&ar, ref_host) == cudaSuccess && as.type == cudaMemoryTypeHost &&
-                    ar.type == cudaMemoryTypeHost && as.devicePointer && ar.devicePointer;
-    (void)cudaGetLastError();
-    if (ok) {
-      s = launch_strip(static_cast<int32_t*>(as.devicePointer), n + 1, static_cast<int64_t>(pair_elems),
-                       static_cast<const int32_t*>(ar.devicePointer), n + 1, static_cast<int64_t>(pair_elems), batch, n, n,
-                       penalty, tile, nullptr, nullptr, 0, 0, hb.st);
-      if (s != NW_OK) return s;
-      NW_CU(cudaStreamSynchronize(hb.st));
-      return NW_OK;
-    }
+  cudaPointerAttributes as{}, ar{};
+  const bool pinned = cudaPointerGetAttributes(&as, score_host) == cudaSuccess &&
+                      cudaPointerGetAttributes(&ar, ref_host) == cudaSuccess && as.type == cudaMemoryTypeHost &&
+                      ar.type == cudaMemoryTypeHost && as.devicePointer && ar.devicePointer;
+  (void)cudaGetLastError();
+  // Pinned (device-mapped) host buffers, zero-copy mode: the kernel streams ref in and score out
+  // over the host link itself (both directions at once, overlapped with the wavefront).
+  if (pinned && g_host_mode == 1) {
+    s = launch_strip(static_cast<int32_t*>(as.devicePointer), n + 1, static_cast<int64_t>(pair_elems),
+                     static_cast<const int32_t*>(ar.devicePointer), n + 1, static_cast<int64_t>(pair_elems), batch, n, n,
+                     penalty, tile, nullptr, nullptr, 0, 0, hb.st);
+    if (s != NW_OK) return s;
+    NW_CU(cudaStreamSynchronize(hb.st));
+    return NW_OK;
   }
+  const bool pipeline = pinned && g_host_mode == 2 && stream_mem_ops();
   std::lock_guard<std::mutex> hlk(g_host_mu[device]);
   {
     std::lock_guard<std::mutex> lk(g_mu);
@@ -552,6 +584,72 @@ nw_status nw_fill_batch_host(int32_t* score_host, const int32_t* ref_host, int64
     }
   }
   const size_t pitch = static_cast<size_t>(n + 1) * 4;
+  if (pipeline) {
+    // Copy-engine pipeline over the stacked matrix's rows (pair * (n+1) + r) in blocks of CHR rows
+    // (~32 MB): the copy-in stream moves the borders, then ref block by block, publishing each
+    // arrival in flags[0] (stream write); the kernel's ref warps wait for the blocks they stage;
+    // its store warps count, per block, the bands whose rows in it are stored (flags[1 + c]); the
+    // copy-out stream waits for each block's count and copies it back.  Both link directions
+    // then run at copy-engine rate while the wavefront runs (zero copy moved ~31 GB/s each way).
+    const int64_t rows = batch * (n + 1);
+    const int64_t chr = g_host_block_rows > 0 ? g_host_block_rows : std::max<int64_t>(64, (int64_t{64} << 20) / static_cast<int64_t>(pitch));
+    const int64_t nblk = (rows + chr - 1) / chr;
+    const int K = tile_to_k(tile);
+    const int64_t nbands = (n + 32 * K - 1) / (32 * K);
+    const int nstore = tile_to_variant(tile) == 1 ? 1 : 2;  // store warps per band (WaveCfg SPB)
+    {
+      std::lock_guard<std::mutex> lk(g_mu);
+      if (!hb.sin) NW_CU(cudaStreamCreateWithFlags(&hb.sin, cudaStreamNonBlocking));
+      if (!hb.sout) NW_CU(cudaStreamCreateWithFlags(&hb.sout, cudaStreamNonBlocking));
+      if (!hb.ev) NW_CU(cudaEventCreateWithFlags(&hb.ev, cudaEventDisableTiming));
+      if (static_cast<size_t>(nblk + 1) > hb.nflags) {
+        if (hb.flags) NW_CU(cudaFree(hb.flags));
+        hb.flags = nullptr;
+        hb.nflags = 0;
+        NW_CU(cudaMalloc(reinterpret_cast<void**>(&hb.flags), static_cast<size_t>(nblk + 1) * 4));
+        hb.nflags = static_cast<size_t>(nblk + 1);
+      }
+    }
+    NW_CU(cudaMemsetAsync(hb.flags, 0, static_cast<size_t>(nblk + 1) * 4, hb.sin));
+    for (int64_t k = 0; k < batch; ++k) {  // borders first: row 0 and column 0 of each pair
+      int32_t* d = hb.score + k * static_cast<int64_t>(pair_elems);
+      const int32_t* h = score_host + k * static_cast<int64_t>(pair_elems);
+      NW_CU(cudaMemcpyAsync(d, h, pitch, cudaMemcpyHostToDevice, hb.sin));
+      NW_CU(cudaMemcpy2DAsync(d + (n + 1), pitch, h + (n + 1), pitch, 4, static_cast<size_t>(n), cudaMemcpyHostToDevice, hb.sin));
+    }
+    NW_CU(cudaEventRecord(hb.ev, hb.sin));
+    NW_CU(cudaStreamWaitEvent(hb.st, hb.ev, 0));
+    NW_CU(cudaStreamWaitEvent(hb.sout, hb.ev, 0));
+    const HostPipe pipe{hb.flags, hb.flags + 1, chr};
+    s = launch_strip(hb.score, n + 1, static_cast<int64_t>(pair_elems), hb.ref, n + 1, static_cast<int64_t>(pair_elems), batch, n,
+                     n, penalty, tile, nullptr, nullptr, 0, 0, hb.st, nullptr, nullptr, 0, 0, nullptr, &pipe);
+    if (s != NW_OK) {
+      (void)cudaStreamSynchronize(hb.sin);
+      return s;
+    }
+    const CUdeviceptr fl = reinterpret_cast<CUdeviceptr>(hb.flags);
+    for (int64_t c = 0; c < nblk; ++c) {
+      const int64_t r0 = c * chr, r1 = std::min(rows, r0 + chr);
+      NW_CU(cudaMemcpyAsync(hb.ref + r0 * (n + 1), ref_host + r0 * (n + 1), static_cast<size_t>(r1 - r0) * pitch,
+                            cudaMemcpyHostToDevice, hb.sin));
+      if (g_write_value(hb.sin, fl, static_cast<cuuint32_t>(c + 1), 0) != CUDA_SUCCESS) return cuda_fail(cudaErrorUnknown);
+    }
+    for (int64_t c = 0; c < nblk; ++c) {
+      const int64_t r0 = c * chr, r1 = std::min(rows, r0 + chr);
+      // signals expected in block c: every band of every pair with an interior row in it
+      const int64_t p_lo = r0 / (n + 1), p_hi = (r1 - 2) / (n + 1);  // pairs with an interior row in [r0, r1)
+      const int64_t npairs = p_hi >= p_lo ? p_hi - p_lo + 1 : 0;
+      const cuuint32_t want = static_cast<cuuint32_t>(npairs * nbands * nstore);
+      if (want > 0 && g_wait_value(hb.sout, fl + 4 * (1 + c), want, CU_STREAM_WAIT_VALUE_GEQ) != CUDA_SUCCESS)
+        return cuda_fail(cudaErrorUnknown);
+      NW_CU(cudaMemcpyAsync(score_host + r0 * (n + 1), hb.score + r0 * (n + 1), static_cast<size_t>(r1 - r0) * pitch,
+                            cudaMemcpyDeviceToHost, hb.sout));
+    }
+    NW_CU(cudaStreamSynchronize(hb.sout));
+    NW_CU(cudaStreamSynchronize(hb.st));
+    NW_CU(cudaStreamSynchronize(hb.sin));
+    return NW_OK;
+  }
   NW_CU(cudaMemcpyAsync(hb.ref, ref_host, elems * 4, cudaMemcpyHostToDevice, hb.st));
   for (int64_t k = 0; k < batch; ++k) {  // borders only: row 0 and column 0 of each pair
     int32_t* d = hb.score + k * static_cast<int64_t>(pair_elems);
@@ -689,7 +787,9 @@ int32_t nw_strip_map(int64_t n, int64_t width, int32_t tile, int32_t band, int32
 void nw_debug_set_grid(int32_t grid) { g_debug_grid = grid > 0 ? grid : 0; }
 void nw_debug_set_pair_mode(int32_t mode) { g_debug_pair_mode = mode < 0 ? -1 : (mode > 0 ? 1 : 0); }
 void nw_debug_set_cluster(int32_t on) { g_debug_cluster = on != 0; }
-void nw_debug_set_host_zero_copy(int32_t on) { g_host_zero_copy = on != 0; }
+void nw_debug_set_host_zero_copy(int32_t on) { g_host_mode = on ? 1 : 2; }
+void nw_debug_set_host_mode(int32_t mode) { g_host_mode = mode < 0 || mode > 2 ? 2 : mode; }
+void nw_debug_set_host_block_rows(int64_t rows) { g_host_block_rows = rows > 0 ? rows : 0; }
 
 void nw_debug_set_trace(uint64_t* dev_buf, int64_t cap_tasks) {
   std::lock_guard<std::mutex> lk(g_mu);

@@ -446,6 +446,8 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
   const bool tracing = kTrace && P.trace2 != nullptr && task < P.trace_cap;
   long long st_busy = 0, st_gap_sum = 0, st_last = tracing ? clock64() : 0;  // (trace) store-warp cycles
   int kr = (SEQ || !DO_REF) ? nch : 0, ks = DO_ST ? max(half, 0) : nch;
+  unsigned rdy = 0;  // host pipeline: cached arrived row blocks
+  long long sig_c = P.rows_done != nullptr ? (g.pair * (P.n + 1) + 1) / P.chunk_rows : 0;  // next block to release
   const uint64_t tw0 = globaltimer_ns();
   uint64_t tw = tw0;
   unsigned idle = 0;
@@ -454,7 +456,16 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
     if (!SEQ && kr < nch) {
       const int need = CH * kr + CH - RR;
       if (consumed < need) prog_read(from_c, consumed, complete);
-      if (consumed >= need) {
+      // host pipeline (nw_fill[_batch]_host): the chunk's ref rows must have arrived; the copy
+      // stream publishes arrived row blocks in *ref_ready (after each copy, stream-ordered)
+      bool arrived = true;
+      if (P.ref_ready != nullptr) {
+        const long long rhi = g.pair * (P.n + 1) + min(n, CH * kr + CH);
+        const unsigned need_c = static_cast<unsigned>(rhi / P.chunk_rows) + 1u;
+        if (rdy < need_c) rdy = ld_acquire_gpu_u32(P.ref_ready);
+        arrived = rdy >= need_c;
+      }
+      if (consumed >= need && arrived) {
         if constexpr (!(NW_DEBUG_SKIP & 5u)) issue_chunk(kr);  // (experiment builds only: results invalid)
         if (kr + C::PFC < nch) prefetch_chunk(kr + C::PFC);
         cp_async_commit();
@@ -470,6 +481,19 @@ __device__ __forceinline__ void wave_stage(const StripParams& P, const long long
         if constexpr (!(NW_DEBUG_SKIP & 9u)) store_chunk(ks);
         if (tracing) st_busy += clock64() - cs0, st_gap_sum += cs0 - st_last, st_last = clock64();
         ks += kstep;
+        if (P.rows_done != nullptr) {
+          // host pipeline: every row block of the stacked matrix below this warp's next chunk is
+          // stored (as far as this warp's chunks go): release it to the device->host copy stream
+          const long long gb = g.pair * (P.n + 1);
+          const long long c_end = ks < nch ? (gb + CH * ks + 1) / P.chunk_rows : (gb + n) / P.chunk_rows + 1;
+          if (sig_c < c_end) {
+            __threadfence();  // this lane's score stores before the counter (gpu scope)
+            __syncwarp();
+            if (t == 0)
+              for (long long c = sig_c; c < c_end; ++c) atomicAdd(P.rows_done + c, 1u);
+            sig_c = c_end;
+          }
+        }
         did = true;
       }
     }

@@ -178,20 +178,31 @@ def test_fill_host_e2e():
     np.testing.assert_array_equal(got, want)
 
 
-@pytest.mark.parametrize("n,tile", [(999, 0), (1500, 64), (3000, 0)])
-def test_fill_host_pinned_zero_copy(n, tile):
-    """Pinned host buffers: the kernel reads ref and writes score over the host link directly."""
+@pytest.mark.parametrize("mode,block_rows", [(1, 0), (0, 0), (2, 0), (2, 37), (2, 256)])
+@pytest.mark.parametrize("n,tile", [(999, 0), (1500, 64), (3000, 0), (1000, 16)])
+def test_fill_host_pinned(n, tile, mode, block_rows):
+    """Pinned host buffers in every host mode: zero copy (the kernel on the host link), staged, and
+    the copy-engine pipeline (ref blocks gated into the kernel, score blocks released back as every
+    band stores them) with automatic, odd and tile-sized row blocks."""
     score, ref = inputs.make_problem(n, 10, seed=23)
     want = expect(score, ref, 10)
     hs = torch.from_numpy(score.copy()).pin_memory()
     hr = torch.from_numpy(ref).pin_memory()
-    nwb.nw_fill_host(hs.numpy(), hr.numpy(), 10, tile, 0)
+    try:
+        nwb.nw_debug_set_host_mode(mode)
+        nwb.nw_debug_set_host_block_rows(block_rows)
+        nwb.nw_fill_host(hs.numpy(), hr.numpy(), 10, tile, 0)
+    finally:
+        nwb.nw_debug_set_host_mode(2)
+        nwb.nw_debug_set_host_block_rows(0)
     np.testing.assert_array_equal(hs.numpy(), want)
 
 
-@pytest.mark.parametrize("pinned", [False, True])
-def test_fill_batch_host(pinned):
-    """Batched end to end from host arrays: staged (pageable) and zero-copy (pinned)."""
+@pytest.mark.parametrize("pinned,mode,block_rows", [(False, 2, 0), (True, 1, 0), (True, 2, 0), (True, 2, 50), (True, 2, 301),
+                                                    (True, 2, 7)])
+def test_fill_batch_host(pinned, mode, block_rows):
+    """Batched end to end from host arrays: staged (pageable), zero copy and the pipeline (pinned),
+    with row blocks inside pairs (50, 7), equal to a pair (301 = n + 1) and automatic."""
     B, n = 5, 300
     ss, rs, want = [], [], []
     for k in range(B):
@@ -201,7 +212,13 @@ def test_fill_batch_host(pinned):
     if pinned:
         St, Rt = torch.from_numpy(S).pin_memory(), torch.from_numpy(R).pin_memory()
         S, R = St.numpy(), Rt.numpy()
-    nwb.nw_fill_batch_host(S, R, 10, 0, 0)
+    try:
+        nwb.nw_debug_set_host_mode(mode)
+        nwb.nw_debug_set_host_block_rows(block_rows)
+        nwb.nw_fill_batch_host(S, R, 10, 0, 0)
+    finally:
+        nwb.nw_debug_set_host_mode(2)
+        nwb.nw_debug_set_host_block_rows(0)
     for k in range(B):
         np.testing.assert_array_equal(S[k], want[k])
 
