@@ -151,7 +151,7 @@ nw_status nw_fill_seq_batch(int32_t* score, int64_t ld_score, int64_t stride_sco
 /* ---- end to end from HOST memory (bench e2e) ---------------------------------------
  * Copies ref (rows 1..n) and the borders host->device, runs nw_fill, copies the full score
  * matrix device->host.  Host buffers: (n+1)x(n+1) int32, pitch n+1.  Pinned buffers take a
- * copy-engine pipeline: ref moves host->device in ~32 MB row blocks on one stream while the
+ * copy-engine pipeline: ref moves host->device in ~64 MB row blocks on one stream while the
  * kernel runs (its ref warps wait for the blocks they stage), and each score row block moves
  * back on a second stream as soon as every band has stored it (stream memory operations on
  * device counters), so both link directions and the wavefront overlap.  Pageable buffers are

@@ -586,7 +586,7 @@ nw_status nw_fill_batch_host(int32_t* score_host, const int32_t* ref_host, int64
   const size_t pitch = static_cast<size_t>(n + 1) * 4;
   if (pipeline) {
     // Copy-engine pipeline over the stacked matrix's rows (pair * (n+1) + r) in blocks of CHR rows
-    // (~32 MB): the copy-in stream moves the borders, then ref block by block, publishing each
+    // (~64 MB): the copy-in stream moves the borders, then ref block by block, publishing each
     // arrival in flags[0] (stream write); the kernel's ref warps wait for the blocks they stage;
     // its store warps count, per block, the bands whose rows in it are stored (flags[1 + c]); the
     // copy-out stream waits for each block's count and copies it back.  Both link directions
