@@ -674,7 +674,7 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
   for (int m = 0; m < K; ++m) Pv[m] = (t * K + m < ws) ? __ldg(g.S + c0 + t * K + m) + (c0 + t * K + m) * p : 0;
   int Lprev = (t * K < ws) ? __ldg(g.S + c0 + t * K - 1) + (c0 + t * K - 1) * p : 0;  // diag input of the first row
   uint64_t e1 = 0ull;                                           // shared source: the next block's entries
-  if constexpr (SRC == kSrcSmem) {
+  if (SRC == kSrcSmem || (SRC == kSrcGlobal && BD == 1)) {
     e1 = load_block(0);
   } else {
     for (int q = 0; q < BD; ++q) prefetch_block(q);
@@ -943,6 +943,8 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
       cur = e1;
       if (sig0 + CE < nsteps) e1 = load_block(Q + 1);
       if (t == 0) sts32_volatile(prog_in, sig0);  // rows <= sig0 consumed (block Q-1 validated)
+    } else if (SRC == kSrcGlobal && BD == 1) {
+      cur = e1;  // the polled producer column: loaded into registers at the previous mid-block
     } else {
       // block Q's copy is in the prologue's group (Q < BD) or in the one committed at the half
       // point of block Q-BD; the groups committed after it may still be in flight
@@ -1001,6 +1003,15 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     // is consumed only there (its latency hides behind the second part's steps instead of
     // stalling the event; measured ~200 cycles per event when read at the event itself)
     auto mid_block = [&]() {
+      if constexpr (SRC == kSrcGlobal) {
+        if (BD == 1) {
+          // a polled producer column: the next block's entries straight into registers (lanes
+          // 0..CE-1, relaxed 8-byte loads, first used at the next event) -- no copy to wait for,
+          // no shared-memory round trip at the event
+          if (sig0 + CE < nsteps) e1 = load_block(Q + 1);
+          return;
+        }
+      }
       if constexpr (SRC != kSrcSmem) {
         // a fresher snapshot of the producer's column than at the event (less band-to-band lag);
         // later than the half point the L2 round trip is exposed at the event
