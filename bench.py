@@ -227,7 +227,8 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--layout", default="rodinia", choices=["rodinia", "aligned"],
-                    help="matrix layout: pitch n+1 (Rodinia) or 16-byte aligned interior rows")
+                    help="device matrix layout: the Rodinia pitch n+1 (default) or 16-byte aligned interior "
+                         "rows (pitch rounded up to 4 elements; 16-byte staging copies)")
     ap.add_argument("--cluster", action="store_true",
                     help="experiment: one pair as thread-block clusters handing the border over through DSMEM")
     ap.add_argument("--trace", default="", help="write per-band {task,start,end,smid} of one extra launch here (.npy)")
@@ -276,8 +277,11 @@ def main():
         from paper_conf_sc_munksgaardhso22_b200 import dist as nwdist
         lo, hi = nwdist.pair_range(B, world, rank)
         nb = hi - lo
-        S = torch.empty((nb, n + 1, n + 1), dtype=torch.int32, device=dev)
-        R = torch.empty((nb, n + 1, n + 1), dtype=torch.int32, device=dev)
+        if args.layout == "aligned":
+            S, R = inputs.device_aligned_batch(nb, n, dev), inputs.device_aligned_batch(nb, n, dev)
+        else:
+            S = torch.empty((nb, n + 1, n + 1), dtype=torch.int32, device=dev)
+            R = torch.empty((nb, n + 1, n + 1), dtype=torch.int32, device=dev)
         for k in range(nb):
             inputs.device_problem(n, p, seed=inputs.pair_seed(lo + k), device=dev, score=S[k], ref=R[k])
 
@@ -357,6 +361,9 @@ def main():
            "config": {"workload": cfg["workload"], "n": n, "batch": B, "penalty": p, "tile": tile,
                       "band_width": nwb.nw_band_width(tile), "pairs_per_rank": B // world if B > 1 else 1,
                       "l2": "inputs %.1f GB >> 126 MB L2 (no flush needed)" % (8.0 * (n + 1) ** 2 * B / 1e9),
+                      "layout": "strips (pitch w+1)" if strips else (
+                          "aligned: interior rows 16-byte aligned, pitch %d" % ((n + 4) & ~3) if args.layout == "aligned"
+                          else "rodinia: pitch n+1"),
                       "parallelism": (f"strips{world}" if strips else f"dp{world}") if world > 1 else "single"},
            "roofline": roof,
            "gpu_launches": args.steps * nwb.nw_launch_count({"strip": 0, "seq": 0, "diagonal": 1, "unopt": 2}[args.variant], n, tile),

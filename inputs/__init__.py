@@ -185,6 +185,15 @@ def device_aligned_matrix(n: int, device="cuda"):
     return buf[3:3 + (n + 1) * ld].view(n + 1, ld)[:, : n + 1]
 
 
+def device_aligned_batch(b: int, n: int, device="cuda"):
+    """A (b, n+1, n+1) int32 CUDA view of b pairs whose interior rows all start 16-byte aligned
+    (pitch and pair stride multiples of 4 elements, element (k, 0, 1) on a 16-byte boundary)."""
+    import torch
+    ld = (n + 1 + 3) & ~3
+    buf = torch.empty(b * (n + 1) * ld + 4, dtype=torch.int32, device=device)
+    return buf[3:3 + b * (n + 1) * ld].view(b, n + 1, ld)[:, :, : n + 1]
+
+
 def device_problem(n: int, p: int = 10, seed: int = SEED, device="cuda", score=None, ref=None,
                    sentinel: bool = True, chunk_rows: int = 4096, layout: str = "rodinia"):
     """The same Rodinia-style problem as make_problem(n, p, seed), built ON THE DEVICE (for the

@@ -62,6 +62,9 @@ namespace nwb200 {
 #ifndef NW_BD_GLOBAL
 #define NW_BD_GLOBAL 1  // border prefetch distance (blocks) of a polled global source
 #endif
+#ifndef NW_PRE_AT
+#define NW_PRE_AT 14  // step at which the next event's staging progress is read (A/B, scripts/gpu_ab.sh)
+#endif
 #ifndef NW_PF_AT
 #define NW_PF_AT 4
 #endif
@@ -751,6 +754,8 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
   // 1..n (no predicates)
   constexpr int kPfAt = NW_PF_AT;  // mid-block work (border copy, progress pre-read) this many steps into the block
   static_assert(kPfAt > 0 && kPfAt < CE, "mid-block point");
+  constexpr int kPreAt = NW_PRE_AT;  // step of the block at which the staging progress is pre-read
+  static_assert(kPreAt >= 0 && kPreAt < CE, "pre-read point");
   // the staging warps' progress words for the NEXT event, read kPfAt steps into the block
   // (the result is first used at that event; cached values that already suffice are kept)
   int cur_sig0 = 0;
@@ -788,7 +793,7 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     // ---- left value: lane t-1's last column of this row, lane 0: the border entry
     const int bval = (ALL && (NW_STEP_EXP & 8)) ? curv + jj : __shfl_sync(FULL, curv, jj);
     const int from_left = (ALL && (NW_STEP_EXP & 128)) ? vlast + 1 : __shfl_up_sync(FULL, vlast, 1);
-    if constexpr (jj == kPfAt) pre_read();  // (its acquire load waits in the shuffles' shadow)
+    if constexpr (jj == kPreAt) pre_read();  // (its acquire load waits in the shuffles' shadow)
     const int L = (ALL && (NW_STEP_EXP & 16)) ? from_left + bval : (t == 0) ? bval : from_left;
     bool active = true;
     if (!ALL) active = r >= 1 && r <= n;
