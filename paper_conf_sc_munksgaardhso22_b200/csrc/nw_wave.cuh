@@ -57,7 +57,7 @@ namespace nwb200 {
 #define NW_RR 128
 #endif
 #ifndef NW_PFC
-#define NW_PFC 12
+#define NW_PFC 4  // L2 prefetch distance of the ref stream, in 8-row chunks (A/B: 3-6 best on config 4, 33.0 vs 34.5 ms at 12; config 3 flat)
 #endif
 #ifndef NW_BD_GLOBAL
 #define NW_BD_GLOBAL 1  // border prefetch distance (blocks) of a polled global source
