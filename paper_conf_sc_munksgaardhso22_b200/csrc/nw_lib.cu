@@ -814,9 +814,15 @@ void nw_release_workspace(void) {
     if (hb.score || hb.ref || hb.st) {
       cudaSetDevice(d);
       if (hb.st) cudaStreamSynchronize(hb.st);
+      if (hb.sin) cudaStreamSynchronize(hb.sin);
+      if (hb.sout) cudaStreamSynchronize(hb.sout);
       if (hb.score) cudaFree(hb.score);
       if (hb.ref) cudaFree(hb.ref);
+      if (hb.flags) cudaFree(hb.flags);
+      if (hb.ev) cudaEventDestroy(hb.ev);
       if (hb.st) cudaStreamDestroy(hb.st);
+      if (hb.sin) cudaStreamDestroy(hb.sin);
+      if (hb.sout) cudaStreamDestroy(hb.sout);
       hb = HostBufs();
     }
   }
