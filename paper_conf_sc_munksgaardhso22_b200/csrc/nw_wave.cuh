@@ -62,6 +62,15 @@ namespace nwb200 {
 #ifndef NW_BD_GLOBAL
 #define NW_BD_GLOBAL 1  // border prefetch distance (blocks) of a polled global source
 #endif
+#ifndef NW_PFC4
+#define NW_PFC4 12  // the same for the K = 4 kernels (tiles 16..128)
+#endif
+#ifndef NW_BORDER_REG
+#define NW_BORDER_REG 1  // polled global border blocks loaded into registers at mid-block (0: cp.async copy)
+#endif
+#ifndef NW_PRE_AT4
+#define NW_PRE_AT4 4
+#endif
 #ifndef NW_PRE_AT
 #define NW_PRE_AT 14  // step at which the next event's staging progress is read (A/B, scripts/gpu_ab.sh)
 #endif
@@ -97,7 +106,7 @@ struct WaveCfg {
   static constexpr int RS = W + 4 * DELTA;      // ring row stride (words)
   static constexpr int RR = NW_RR;               // ref ring rows (the staging warp's lookahead)
   static constexpr int SR = 64;                 // score ring rows
-  static constexpr int PFC = NW_PFC;            // L2 prefetch distance (chunks of CH rows) of the staging warp
+  static constexpr int PFC = K == 8 ? NW_PFC : NW_PFC4;  // L2 prefetch distance (chunks of CH rows) of the staging warp
   static constexpr int BR = 256;                // shared border ring entries
   static constexpr int NL = (4 * W + 127) / 128 + 1;  // 128-byte lines touched by one row segment
   static constexpr int REF_WORDS = SEQ ? 0 : RR * RS;
@@ -677,7 +686,7 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
   for (int m = 0; m < K; ++m) Pv[m] = (t * K + m < ws) ? __ldg(g.S + c0 + t * K + m) + (c0 + t * K + m) * p : 0;
   int Lprev = (t * K < ws) ? __ldg(g.S + c0 + t * K - 1) + (c0 + t * K - 1) * p : 0;  // diag input of the first row
   uint64_t e1 = 0ull;                                           // shared source: the next block's entries
-  if (SRC == kSrcSmem || (SRC == kSrcGlobal && BD == 1)) {
+  if (SRC == kSrcSmem || (SRC == kSrcGlobal && BD == 1 && NW_BORDER_REG)) {
     e1 = load_block(0);
   } else {
     for (int q = 0; q < BD; ++q) prefetch_block(q);
@@ -754,7 +763,9 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
   // 1..n (no predicates)
   constexpr int kPfAt = NW_PF_AT;  // mid-block work (border copy, progress pre-read) this many steps into the block
   static_assert(kPfAt > 0 && kPfAt < CE, "mid-block point");
-  constexpr int kPreAt = NW_PRE_AT;  // step of the block at which the staging progress is pre-read
+  // step of the block at which the staging progress is pre-read (A/B: late for the K = 8 kernel,
+  // early for the K = 4 kernels, whose two-band CTA measured 235 vs 204 GCUPS at 4 vs 14)
+  constexpr int kPreAt = K == 8 ? NW_PRE_AT : NW_PRE_AT4;
   static_assert(kPreAt >= 0 && kPreAt < CE, "pre-read point");
   // the staging warps' progress words for the NEXT event, read kPfAt steps into the block
   // (the result is first used at that event; cached values that already suffice are kept)
@@ -948,7 +959,7 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
       cur = e1;
       if (sig0 + CE < nsteps) e1 = load_block(Q + 1);
       if (t == 0) sts32_volatile(prog_in, sig0);  // rows <= sig0 consumed (block Q-1 validated)
-    } else if (SRC == kSrcGlobal && BD == 1) {
+    } else if (SRC == kSrcGlobal && BD == 1 && NW_BORDER_REG) {
       cur = e1;  // the polled producer column: loaded into registers at the previous mid-block
     } else {
       // block Q's copy is in the prologue's group (Q < BD) or in the one committed at the half
@@ -1008,7 +1019,7 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
     // is consumed only there (its latency hides behind the second part's steps instead of
     // stalling the event; measured ~200 cycles per event when read at the event itself)
     auto mid_block = [&]() {
-      if constexpr (SRC == kSrcGlobal) {
+      if constexpr (SRC == kSrcGlobal && NW_BORDER_REG) {
         if (BD == 1) {
           // a polled producer column: the next block's entries straight into registers (lanes
           // 0..CE-1, relaxed 8-byte loads, first used at the next event) -- no copy to wait for,
