@@ -345,7 +345,10 @@ def main():
     achieved = bpc * cells_local / (kern_ms * 1e-3) / 1e9
     peak, peak_src = measured_peaks()
     roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-            "traffic": ncu_traffic(cfg["workload"], tile), "peak_source": peak_src,
+            "traffic": ncu_traffic(cfg["workload"], tile),
+            "traffic_source": "profiles/ncu_traffic.json: dram__bytes_read.sum + dram__bytes_write.sum per launch "
+                              "from the latest ncu --set full capture of this kernel (profiles/r02c_*)",
+            "peak_source": peak_src,
             "algorithmic_bytes_per_launch": int(bpc * cells_local),
             "kernel": ("nw_wave_kernel<WaveCfg<K=%d, SEQ=%d>> (W = %d columns per band)"
                        % (nwb.nw_band_width(tile) // 32, int(args.variant == "seq"), nwb.nw_band_width(tile)))
