@@ -22,24 +22,31 @@
 //         word 32i+t: the copy realigns the row whatever its 16-byte phase, which the Rodinia
 //         pitch n+1 changes from row to row), 8-row chunks, plus an L2 prefetch further ahead;
 //       - score rows: K LDS.32 + K coalesced STG.32 per lane and row.
-//     Ring row x of row r is (r-1) & 63; the row stride RS = W + 4*delta words shifts the
+//     Ring row x of row r is (r-1) & (RR-1) (ref) / (r-1) & 63 (score); the row stride RS = W + 4*delta words shifts the
 //     16-byte bank group by delta per row, which makes the skewed LDS/STS.128 of the 32 lanes
 //     (32 different rows) conflict free (K=8: delta=1, K=4: delta=2).
 //     The two warps synchronise through two 64-bit progress words in shared memory (release /
 //     acquire, polled only when the cached value is insufficient): compute -> staging {ref rows
 //     consumed, score rows complete}, staging -> compute {ref rows landed, score rows stored}.
-//   * Compute-warp events every CH = 8 steps: progress words, border-block check (+ its cp.async
-//     commit / wait), back-pressure, __syncwarp.  No other synchronisation inside a band.
+//   * Compute-warp events every CE = 16 steps (blocks fully unrolled, border-lane indices
+//     immediates): publish the progress word, compare the staging progress read 14 steps into the
+//     previous block (in a shuffle's shadow; re-read and spin only if short), take the border
+//     block, back-pressure on a shared sink.  No other synchronisation inside a band.
 //   * Band handoff (the paper's Fig. 9 ordering W ∩ R = ∅): the lane holding the band's last
-//     column publishes every row as a 64-bit entry {value, tag} (flag fused with the value):
+//     column publishes every row as a 64-bit entry {value, tag} (flag fused with the value;
+//     steady blocks publish 8 rows at a time as four 16-byte pairs):
 //       - to warp w+1 of the CTA: a 256-entry shared ring (tag = gen << 30 | row), back-pressure
 //         on the consumer's published progress;
 //       - to another CTA / GPU: a full-length global buffer (tag = launch epoch), relaxed
 //         gpu / sys scope stores.
-//     The consumer holds one 8-row block of entries per event (lanes 0..7); global / plain
-//     sources are copied three blocks ahead by cp.async into a small shared ring (no register
-//     holds an in-flight load across an event), a shared source is read one block ahead; a
+//     The consumer holds one 16-row block of entries per event (lanes 0..15): a polled producer
+//     column is loaded into registers 4 steps into the previous block (relaxed 8-byte loads); a
+//     complete one (the input column, or in pair mode a finished band) is copied three blocks
+//     ahead by cp.async into a small shared ring; a shared source is read one block ahead.  A
 //     stale block is re-polled synchronously under a %globaltimer watchdog (trap on expiry).
+//   * Layouts whose interior rows are 16-byte aligned stage with 16-byte copies / stores
+//     (StripParams::vec16).  The host pipeline (nw_fill[_batch]_host) gates the ref warp on
+//     arrived row blocks and counts stored row blocks for the copy-out stream.
 #pragma once
 #include <cstdint>
 #include <utility>
