@@ -769,7 +769,7 @@ __device__ __forceinline__ void wave_band(const StripParams& P, const long long 
   // one wavefront step s (entry jj of the block's border window); ALL = every lane's row is in
   // 1..n (no predicates)
   constexpr int kPfAt = NW_PF_AT;  // mid-block work (border copy, progress pre-read) this many steps into the block
-  static_assert(kPfAt > 0 && kPfAt < CE, "mid-block point");
+  static_assert(kPfAt >= 0 && kPfAt < CE, "mid-block point");
   // step of the block at which the staging progress is pre-read (A/B: late for the K = 8 kernel,
   // early for the K = 4 kernels, whose two-band CTA measured 235 vs 204 GCUPS at 4 vs 14)
   constexpr int kPreAt = K == 8 ? NW_PRE_AT : NW_PRE_AT4;
